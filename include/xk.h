@@ -1,0 +1,267 @@
+/*
+ * xk.h -- C ABI of the B200-native XKBlas-style multi-GPU level-3 BLAS (libxk.so).
+ *
+ * The method (Gautier & Lima, PAW-ATM/SC21, /root/reference/PAPER.md):
+ *   - LAPACK-layout (column-major) BLAS-3 split into tile tasks on sub-matrix views
+ *     (§III, §III-A "memory view" / compact device tile),
+ *   - owner-computes mapping of tasks, here a static 2D block-cyclic P x Q
+ *     grid,
+ *   - a per-tile coherence directory of valid copies on host and GPUs,
+ *   - source selection for every input tile by two heuristics:
+ *       (i)  topology-aware: among GPUs holding a valid copy, prefer the best link
+ *            toward the destination (§III-B),
+ *       (ii) optimistic forwarding: when no GPU holds a valid copy, take the best GPU
+ *            whose copy is still in flight instead of the host (§III-C),
+ *   - lazy host coherence: results stay on the GPUs until the user asks for them
+ *     (xkblas_memory_coherent_async),
+ *   - asynchronous calls that compose through the cache.
+ *
+ * Conventions:
+ *   - All matrices are column-major host arrays owned by the caller; dimensions and
+ *     leading dimensions are int64_t.  Char arguments are case-insensitive; 'C' == 'T'.
+ *   - Return value: 0 on success; -i when argument i is invalid (numbered like the
+ *     reference BLAS XERBLA, in argument order); a positive XK_ERR_* on runtime failure.
+ *     The library never aborts; xk_last_error() returns a message for the last failure.
+ *   - BLAS "not referenced" rules hold: beta == 0 -> C is not read (and not copied to a
+ *     GPU); alpha == 0 -> A, B not read; quick return when m == 0, n == 0 or
+ *     ((alpha == 0 || k == 0) && beta == 1); rows beyond m in ld-padded storage are
+ *     never written.
+ *   - Synchronous routines = async + coherence of the output + wait + invalidation of
+ *     the device copies of their operands (drop-in semantics).
+ *     Asynchronous routines return as soon as the work is issued; inputs must stay
+ *     unmodified and outputs unread until xk_memory_coherent_sync() on that view (or
+ *     xk_sync() followed by coherence).  Device copies stay in the library cache, so a
+ *     following async call reads them from the GPUs (composition).
+ *   - Calls must come from one host thread at a time (an internal mutex serialises).
+ *   - Host memory should be registered with xk_register() before timed calls
+ *     (page-locking is excluded from the paper's timings); unregistered
+ *     memory is registered internally on first use and counted in the stats.
+ */
+#ifndef XK_H
+#define XK_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ------------------------------------------------------------------ error codes */
+#define XK_OK 0
+#define XK_ERR_NOT_INITIALIZED 1 /* xk_init() not called */
+#define XK_ERR_CUDA 2            /* a CUDA runtime/driver call failed; see xk_last_error() */
+#define XK_ERR_OOM 3             /* device tile cache full (no eviction: SURVEY A13) */
+#define XK_ERR_CONFIG 4          /* invalid xk_config_t / topology / flags */
+#define XK_ERR_CAPACITY 5        /* caller-provided output array too small */
+#define XK_ERR_UNSUPPORTED 6     /* view overlaps a cached matrix with another tiling */
+#define XK_ERR_NO_DEVICE 7       /* no CUDA device visible */
+#define XK_ERR_INTERNAL 8
+
+#define XK_MAX_GPUS 16
+#define XK_HOST (-1) /* node id of host memory in plan records */
+
+/* topology-aware source selection modes (a5) */
+#define XK_TOPO_RANKED 0   /* paper's heuristic: best link class first */
+#define XK_TOPO_UNRANKED 1 /* paper's "no topo" ablation: lowest-index holder */
+#define XK_TOPO_HOME 2     /* link-oblivious ablation: host first, then GPUs */
+
+/* ------------------------------------------------------------------ configuration */
+typedef struct xk_config {
+    int ngpus;            /* logical GPUs G (0 = every visible device, max XK_MAX_GPUS) */
+    int phys[XK_MAX_GPUS];/* logical -> physical device map; used when map_devices != 0,
+                             else logical g -> physical g mod device_count.  Several
+                             logical GPUs on one physical device = "logical-device mode"
+                             (peer copies become device-to-device copies). */
+    int map_devices;
+    int grid_p, grid_q;   /* owner grid P x Q (0,0 = near-square P >= Q: 1x1,2x1,2x2,4x2) */
+    int64_t tile;         /* tile size T (0 = 2048) */
+    int topo;             /* XK_TOPO_* (default RANKED) */
+    int optimistic;       /* optimistic forwarding on (1, default) / off (0) */
+    int window;           /* planner prefetch window W in tasks (0 = 2) */
+    int kstreams;         /* kernel streams per GPU (0 = 2); plus 1 H2D, 1 D2H, 1 P2P-in */
+    int probe;            /* 1 = time the (G+1)^2 link matrix at init (a1); 0 = defaults */
+    int64_t task_rate_mflops; /* planner's tile-task rate (0 = derived from the FP64 peak) */
+} xk_config_t;
+
+/* Fill *cfg with defaults, then apply the environment (XK_NGPUS, XK_TILE,
+ * XK_TOPO=ranked|unranked|home, XK_OPTIMISTIC=0|1, XK_WINDOW, XK_KSTREAMS, XK_PROBE). */
+void xk_config_default(xk_config_t *cfg);
+
+/* ------------------------------------------------------------------ lifecycle */
+int xk_init(const xk_config_t *cfg); /* NULL -> xk_config_default(); probes topology */
+int xk_finalize(void);               /* waits, frees every device copy, destroys streams */
+int xk_register(void *p, size_t bytes);   /* cudaHostRegister(Portable) once, all GPUs */
+int xk_unregister(void *p);
+const char *xk_last_error(void);
+
+/* ------------------------------------------------------------------ BLAS-3 (FP64) */
+/* C <- alpha*op(A)*op(B) + beta*C ; op(X) = X ('N') or X^T ('T'/'C').
+ * A is m x k ('N') or k x m ('T') with lda >= max(1, rows); B is k x n or n x k; C m x n.
+ * Errors: -1 transA, -2 transB, -3 m, -4 n, -5 k, -8 lda, -10 ldb, -13 ldc. */
+int xk_dgemm(char transA, char transB, int64_t m, int64_t n, int64_t k, double alpha,
+             const double *A, int64_t lda, const double *B, int64_t ldb,
+             double beta, double *C, int64_t ldc);
+int xk_dgemm_async(char transA, char transB, int64_t m, int64_t n, int64_t k, double alpha,
+                   const double *A, int64_t lda, const double *B, int64_t ldb,
+                   double beta, double *C, int64_t ldc);
+
+/* C <- alpha*op(A)*op(A)^T + beta*C on the uplo triangle only (op(A) n x k).
+ * Errors: -1 uplo, -2 trans, -3 n, -4 k, -7 lda, -10 ldc. */
+int xk_dsyrk(char uplo, char trans, int64_t n, int64_t k, double alpha,
+             const double *A, int64_t lda, double beta, double *C, int64_t ldc);
+int xk_dsyrk_async(char uplo, char trans, int64_t n, int64_t k, double alpha,
+                   const double *A, int64_t lda, double beta, double *C, int64_t ldc);
+
+/* C <- alpha*op(A)*op(B)^T + alpha*op(B)*op(A)^T + beta*C, uplo triangle only.
+ * Errors: -1 uplo, -2 trans, -3 n, -4 k, -7 lda, -9 ldb, -12 ldc. */
+int xk_dsyr2k(char uplo, char trans, int64_t n, int64_t k, double alpha,
+              const double *A, int64_t lda, const double *B, int64_t ldb,
+              double beta, double *C, int64_t ldc);
+int xk_dsyr2k_async(char uplo, char trans, int64_t n, int64_t k, double alpha,
+                    const double *A, int64_t lda, const double *B, int64_t ldb,
+                    double beta, double *C, int64_t ldc);
+
+/* C <- alpha*sym(A)*B + beta*C ('L') or alpha*B*sym(A) + beta*C ('R'); only the uplo
+ * triangle of A is read.  Errors: -1 side, -2 uplo, -3 m, -4 n, -7 lda, -9 ldb, -12 ldc. */
+int xk_dsymm(char side, char uplo, int64_t m, int64_t n, double alpha,
+             const double *A, int64_t lda, const double *B, int64_t ldb,
+             double beta, double *C, int64_t ldc);
+int xk_dsymm_async(char side, char uplo, int64_t m, int64_t n, double alpha,
+                   const double *A, int64_t lda, const double *B, int64_t ldb,
+                   double beta, double *C, int64_t ldc);
+
+/* B <- alpha*op(A)*B ('L') or alpha*B*op(A) ('R'), A triangular (uplo), diag 'U' = unit.
+ * Errors: -1 side, -2 uplo, -3 transA, -4 diag, -5 m, -6 n, -9 lda, -11 ldb. */
+int xk_dtrmm(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
+             double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
+int xk_dtrmm_async(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
+                   double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
+
+/* Solve op(A)*X = alpha*B ('L') or X*op(A) = alpha*B ('R'); B <- X.  Same errors as TRMM. */
+int xk_dtrsm(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
+             double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
+int xk_dtrsm_async(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
+                   double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
+
+/* ------------------------------------------------------------------ coherence / sync */
+/* Make the host view (m x n at A, leading dimension lda) coherent: copy back every
+ * cached tile intersection whose host copy is stale (only the intersection is written),
+ * after its last writer.  _sync blocks until done. */
+int xk_memory_coherent_sync(int64_t m, int64_t n, double *A, int64_t lda);
+int xk_memory_coherent_async(int64_t m, int64_t n, double *A, int64_t lda);
+/* Wait for all issued work.  Does NOT make host copies coherent (lazy). */
+int xk_sync(void);
+/* Drop the device copies of the tiles of a view (waits for pending work first).
+ * Stale host tiles are NOT written back: call xk_memory_coherent_sync first. */
+int xk_memory_invalidate(int64_t m, int64_t n, const double *A, int64_t lda);
+/* Load the tiles of a host view onto their owner GPUs now (data-on-device runs). */
+int xk_memory_prefetch_async(int64_t m, int64_t n, const double *A, int64_t lda);
+
+/* ------------------------------------------------------------------ observability */
+typedef struct xk_stats {
+    int ngpus;
+    int64_t h2d_bytes[XK_MAX_GPUS];  /* host -> GPU g */
+    int64_t d2h_bytes[XK_MAX_GPUS];  /* GPU g -> host */
+    int64_t p2p_in_bytes[XK_MAX_GPUS];  /* peer -> GPU g */
+    int64_t p2p_out_bytes[XK_MAX_GPUS]; /* GPU g -> peer */
+    int64_t tasks[XK_MAX_GPUS];
+    int64_t flops[XK_MAX_GPUS];
+    int64_t forwards_inflight;       /* P2P copies sourced from an in-flight copy (A2) */
+    int64_t forwards_valid;          /* P2P copies sourced from a valid copy (A1) */
+    int64_t kernel_launches;
+    int64_t host_registrations;      /* unregistered host ranges registered internally */
+    double kernel_ms_total;          /* summed dgemm tile-kernel time (when timing on) */
+} xk_stats_t;
+int xk_get_stats(xk_stats_t *out);
+int xk_reset_stats(void);
+/* 1 = time every tile kernel with CUDA events (bench roofline); 0 = off (default). */
+int xk_set_kernel_timing(int on);
+
+/* (G+1) x (G+1) link matrix in MB/s, row = source, column = destination, index G =
+ * host; diagonal = device-local copy bandwidth.  Filled by xk_init (probe or defaults). */
+typedef struct xk_topo {
+    int ngpus;
+    int64_t bw_MBps[(XK_MAX_GPUS + 1) * (XK_MAX_GPUS + 1)]; /* row-major, stride ngpus+1 */
+    int perf_rank[XK_MAX_GPUS * XK_MAX_GPUS]; /* cuDeviceGetP2PAttribute PERFORMANCE_RANK, logged only (Q6) */
+    int64_t task_rate_mflops;                 /* tile-task FP64 rate used by the planner */
+} xk_topo_t;
+int xk_get_topology(xk_topo_t *out);
+
+/* ------------------------------------------------------------------ planner (no GPU) */
+/* The planner is a pure function of (call, topology, flags, directory state): tests run
+ * it with G virtual GPUs and injected link matrices and compare it bit-exactly with the
+ * independent CPU model tests/planmodel.py (SURVEY.md §8(c) "Plan oracle"). */
+#define XK_REC_H2D 0
+#define XK_REC_P2P 1
+#define XK_REC_TASK 2
+#define XK_REC_D2H 3
+
+#define XK_SRC_NONE 0
+#define XK_SRC_VALID 1    /* source copy valid at request time */
+#define XK_SRC_INFLIGHT 2 /* source copy still arriving: optimistic forwarding */
+#define XK_SRC_HOST 3
+
+#define XK_ROUTINE_DGEMM 0
+#define XK_ROUTINE_COHERENT 100
+#define XK_ROUTINE_SYNC 101
+#define XK_ROUTINE_INVALIDATE 102
+#define XK_ROUTINE_PREFETCH 103
+
+typedef struct xk_flags {
+    int topo, optimistic, window;
+    int grid_p, grid_q;
+    int64_t tile;
+} xk_flags_t;
+
+/* One API call as seen by the planner.  Matrix addresses are identities only (never
+ * dereferenced by the planner).  For XK_ROUTINE_COHERENT / INVALIDATE the view is
+ * (m, n, C, ldc). */
+typedef struct xk_call {
+    int routine;
+    char transA, transB;
+    int64_t m, n, k;
+    double alpha, beta;
+    uint64_t A, lda, B, ldb, C, ldc;
+    int sync; /* 1 = synchronous routine: D2H of the output after its last writer */
+} xk_call_t;
+
+typedef struct xk_plan_rec {
+    int64_t seq;       /* emission order, session-global */
+    int32_t kind;      /* XK_REC_* */
+    int32_t operand;   /* 0 = A, 1 = B, 2 = C of the call (coherent/prefetch: 2) */
+    int64_t bi, bj;    /* tile coordinates in the STORED matrix (T x T grid at element 0,0) */
+    int64_t tk;        /* TASK: k-tile index (-1: scale-only task C <- beta*C) */
+    int64_t version;   /* tile version the record moves / produces */
+    int32_t dst, src;  /* node ids: GPU 0..G-1 or XK_HOST */
+    int32_t src_state; /* XK_SRC_* (copies); XK_SRC_NONE for tasks */
+    int32_t depth;     /* forwarding depth of the destination copy (host = 0, H2D = 1) */
+    int64_t t_start, t_end; /* virtual time, integer ns */
+    int64_t work;      /* bytes (copies) or flops (tasks) */
+    int64_t dep[4];    /* seq of records this one waits on (-1 = none) */
+} xk_plan_rec_t;
+
+/* Planner sessions: the directory, clocks and link occupancy persist across calls
+ * (composition), exactly as inside the library. */
+typedef struct xk_plan_session xk_plan_session_t;
+int xk_plan_session_create(const xk_topo_t *topo, const xk_flags_t *flags, xk_plan_session_t **out);
+int xk_plan_session_call(xk_plan_session_t *s, const xk_call_t *call,
+                         xk_plan_rec_t *out, int64_t cap, int64_t *n_out);
+void xk_plan_session_destroy(xk_plan_session_t *s);
+/* One-shot: fresh session, one call. */
+int xk_plan_dump(const xk_call_t *call, const xk_topo_t *topo, const xk_flags_t *flags,
+                 xk_plan_rec_t *out, int64_t cap, int64_t *n_out);
+
+/* ------------------------------------------------------------------ kernel-level entry */
+/* One tile task on device memory, for kernel parity tests and the roofline bench:
+ * D = alpha*op(A)*op(B) + beta*C on compact column-major tiles (ld = rows),
+ * D may alias C.  Pointers are DEVICE pointers on the current device; stream is a
+ * cudaStream_t (NULL = legacy default stream).  beta == 0: C not read. */
+int xk_dgemm_tile_device(char transA, char transB, int64_t m, int64_t n, int64_t k,
+                         double alpha, const double *A, int64_t lda, const double *B,
+                         int64_t ldb, double beta, double *C, int64_t ldc, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* XK_H */

@@ -1,0 +1,605 @@
+// plan.cpp -- see plan.h.  Every numbered step below refers to SURVEY.md §8(c)
+// "Plan oracle" (the readings are restated in DESIGN.md §Readings); the CPU model in
+// tests/planmodel.py implements the same steps independently and must agree bit for bit.
+#include "plan/plan.h"
+
+#include <algorithm>
+#include <cstring>
+#include <map>
+#include <tuple>
+
+namespace xk {
+
+static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+std::vector<int> link_classes(int G, const std::vector<int64_t> &bw) {
+    // step 1: sort the off-diagonal bandwidths; a new class starts whenever consecutive
+    // distinct values differ by a ratio > 1.25 (4*v[i] > 5*v[i-1]); higher = faster.
+    const int N = G + 1;
+    std::vector<int64_t> v;
+    for (int s = 0; s < N; ++s)
+        for (int d = 0; d < N; ++d)
+            if (s != d) v.push_back(bw[(size_t)s * N + d]);
+    std::sort(v.begin(), v.end());
+    v.erase(std::unique(v.begin(), v.end()), v.end());
+    std::map<int64_t, int> cls_of;
+    int c = 0;
+    for (size_t i = 0; i < v.size(); ++i) {
+        if (i > 0 && 4 * v[i] > 5 * v[i - 1]) ++c;
+        cls_of[v[i]] = c;
+    }
+    std::vector<int> cls((size_t)N * N, 1 << 20);
+    for (int s = 0; s < N; ++s)
+        for (int d = 0; d < N; ++d)
+            if (s != d) cls[(size_t)s * N + d] = cls_of[bw[(size_t)s * N + d]];
+    return cls;
+}
+
+Planner::Planner(const Topology &t, const Flags &f) : topo_(t), flags_(f) {
+    cls_ = link_classes(t.G, t.bw);
+    link_free_.assign((size_t)(t.G + 1) * (t.G + 1), 0);
+    gpu_free_.assign(t.G, 0);
+    ends_.assign(t.G, {});
+}
+
+int64_t Planner::dur(int64_t amount, int64_t rate) const {
+    // copies: ceil(bytes*1000 / MBps) ns; tasks: ceil(flops*1000 / MFLOPs) ns (step 3, 5)
+    return cdiv(amount * 1000, rate);
+}
+
+int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t cols,
+                                std::string &err) {
+    for (size_t i = 0; i < mats_.size(); ++i) {
+        Matrix &M = mats_[i];
+        if (M.ld < 0) continue;  // forgotten
+        if (M.base == base && M.ld == ld) {
+            // tile extents must agree with the cached grid (step 9)
+            int64_t T = flags_.T;
+            auto edge_ok = [&](int64_t a, int64_t b) {
+                // same ragged edge tile or both multiples beyond the shorter extent
+                int64_t lo = std::min(a, b), hi = std::max(a, b);
+                if (lo == hi) return true;
+                return lo % T == 0 && cdiv(lo, T) <= cdiv(hi, T);
+            };
+            if (!edge_ok(M.rows, rows) || !edge_ok(M.cols, cols)) {
+                // a clean matrix (no GPU copies, host valid) can simply be forgotten
+                bool clean = true;
+                for (auto &kv : keymap_) {
+                    const Entry &e = entries_[kv.second];
+                    if (e.mat != (int)i) continue;
+                    for (auto &g : e.gpu) clean = clean && !g.present;
+                    clean = clean && e.host.present && e.host.ver == e.ver;
+                }
+                if (!clean) {
+                    err = "view of a cached matrix with a different tiling (make it coherent and invalidate first)";
+                    return -1;
+                }
+                for (auto it = keymap_.begin(); it != keymap_.end();)
+                    if (entries_[it->second].mat == (int)i) it = keymap_.erase(it); else ++it;
+                M.rows = rows;
+                M.cols = cols;
+                return (int)i;
+            }
+            M.rows = std::max(M.rows, rows);
+            M.cols = std::max(M.cols, cols);
+            return (int)i;
+        }
+    }
+    // overlap with another cached matrix at a different anchor -> unsupported unless clean
+    uint64_t lo = base, hi = base + (uint64_t)((cols - 1) * ld + rows) * 8;
+    for (size_t i = 0; i < mats_.size(); ++i) {
+        Matrix &M = mats_[i];
+        if (M.ld < 0) continue;
+        uint64_t mlo = M.base, mhi = M.base + (uint64_t)((M.cols - 1) * M.ld + M.rows) * 8;
+        if (lo < mhi && mlo < hi) {
+            bool clean = true;
+            for (auto &kv : keymap_) {
+                const Entry &e = entries_[kv.second];
+                if (e.mat != (int)i) continue;
+                for (auto &g : e.gpu) clean = clean && !g.present;
+                clean = clean && e.host.present && e.host.ver == e.ver;
+            }
+            if (!clean) {
+                err = "view overlaps a cached matrix anchored elsewhere (make it coherent and invalidate first)";
+                return -1;
+            }
+            for (auto it = keymap_.begin(); it != keymap_.end();)
+                if (entries_[it->second].mat == (int)i) it = keymap_.erase(it); else ++it;
+            M.ld = -1;  // forget
+        }
+    }
+    Matrix M;
+    M.base = base;
+    M.ld = ld;
+    M.rows = rows;
+    M.cols = cols;
+    mats_.push_back(M);
+    return (int)mats_.size() - 1;
+}
+
+int Planner::key_of(int mat, int64_t bi, int64_t bj) {
+    std::string k(sizeof(int) + 2 * sizeof(int64_t), '\0');
+    std::memcpy(&k[0], &mat, sizeof(int));
+    std::memcpy(&k[sizeof(int)], &bi, sizeof(int64_t));
+    std::memcpy(&k[sizeof(int) + sizeof(int64_t)], &bj, sizeof(int64_t));
+    auto it = keymap_.find(k);
+    if (it != keymap_.end()) return it->second;
+    Entry e;
+    e.mat = mat;
+    e.bi = bi;
+    e.bj = bj;
+    const Matrix &M = mats_[mat];
+    e.rows = std::min(flags_.T, M.rows - bi * flags_.T);
+    e.cols = std::min(flags_.T, M.cols - bj * flags_.T);
+    e.ver = 0;
+    e.host.present = true;  // inputs start VALID on the host (step 4)
+    e.host.ver = 0;
+    e.gpu.assign(topo_.G, NodeCopy());
+    entries_.push_back(e);
+    int id = (int)entries_.size() - 1;
+    keymap_[k] = id;
+    return id;
+}
+
+// step 4: source selection for a tile needed on GPU d at request time treq.
+int Planner::select_source(const Entry &e, int64_t ver, int d, int64_t treq, int *state) const {
+    const int G = topo_.G;
+    std::vector<int> V, I;
+    for (int g = 0; g < G; ++g) {
+        if (g == d) continue;
+        const NodeCopy &c = e.gpu[g];
+        if (!c.present || c.ver != ver) continue;
+        if (c.t_done <= treq) V.push_back(g); else I.push_back(g);
+    }
+    bool host_ok = e.host.present && e.host.ver == ver;
+    auto ranked_best = [&](const std::vector<int> &L) {
+        int best = -1;
+        std::tuple<int, int, int> bk;
+        for (int g : L) {
+            std::tuple<int, int, int> k(-cls_[(size_t)g * (G + 1) + d], e.gpu[g].depth,
+                                        ((g - d) % G + G) % G);
+            if (best < 0 || k < bk) { best = g; bk = k; }
+        }
+        return best;
+    };
+    auto lowest = [&](const std::vector<int> &L) { return L.empty() ? -1 : L.front(); };
+    int mode = flags_.topo;
+    if (mode == XK_TOPO_HOME) {
+        if (host_ok) { *state = XK_SRC_HOST; return XK_HOST; }
+        if (!V.empty()) { *state = XK_SRC_VALID; return lowest(V); }
+        if (!I.empty()) { *state = XK_SRC_INFLIGHT; return lowest(I); }
+        *state = XK_SRC_NONE;
+        return -2;
+    }
+    auto pick = [&](const std::vector<int> &L) {
+        return mode == XK_TOPO_RANKED ? ranked_best(L) : lowest(L);
+    };
+    if (!V.empty()) { *state = XK_SRC_VALID; return pick(V); }
+    if (!I.empty() && (flags_.optimistic || !host_ok)) { *state = XK_SRC_INFLIGHT; return pick(I); }
+    if (host_ok) { *state = XK_SRC_HOST; return XK_HOST; }
+    *state = XK_SRC_NONE;
+    return -2;
+}
+
+// step 5: copy timing, store-and-forward after the source copy completes.
+bool Planner::emit_copy(int key, int64_t ver, int d, int64_t treq, int operand,
+                        std::vector<Rec> &out) {
+    Entry &e = entries_[key];
+    const int G = topo_.G;
+    int state = 0;
+    int src = select_source(e, ver, d, treq, &state);
+    if (src == -2) return false;  // no copy of this version anywhere (lost by invalidate)
+    int sidx = (src == XK_HOST) ? G : src;
+    int64_t bytes = 8 * e.rows * e.cols;
+    int64_t src_ready, dep;
+    int depth;
+    if (src == XK_HOST) {
+        src_ready = e.host.t_done;
+        dep = e.host.producer;
+        depth = 1;
+    } else {
+        src_ready = e.gpu[src].t_done;
+        dep = e.gpu[src].producer;
+        depth = e.gpu[src].depth + 1;
+    }
+    int64_t &lf = link_free_[(size_t)sidx * (G + 1) + d];
+    int64_t t0 = std::max(treq, std::max(src_ready, lf));
+    int64_t t1 = t0 + dur(bytes, topo_.bw_at(sidx, d));
+    lf = t1;
+    Rec R;
+    std::memset(&R.r, 0, sizeof(R.r));
+    R.r.seq = seq_++;
+    R.r.kind = (src == XK_HOST) ? XK_REC_H2D : XK_REC_P2P;
+    R.r.operand = operand;
+    R.r.bi = e.bi;
+    R.r.bj = e.bj;
+    R.r.tk = -1;
+    R.r.version = ver;
+    R.r.dst = d;
+    R.r.src = src;
+    R.r.src_state = state;
+    R.r.depth = depth;
+    R.r.t_start = t0;
+    R.r.t_end = t1;
+    R.r.work = bytes;
+    R.r.dep[0] = dep;
+    R.r.dep[1] = R.r.dep[2] = R.r.dep[3] = -1;
+    R.key = key;
+    R.sub_rows = e.rows;
+    R.sub_cols = e.cols;
+    out.push_back(R);
+    NodeCopy &c = e.gpu[d];
+    c.present = true;
+    c.ver = ver;
+    c.t_done = t1;
+    c.producer = R.r.seq;
+    c.depth = depth;
+    return true;
+}
+
+void Planner::emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, int64_t cols,
+                       int64_t ready, int64_t dep, int operand, std::vector<Rec> &out) {
+    Entry &e = entries_[key];
+    const int G = topo_.G;
+    int64_t bytes = 8 * rows * cols;
+    int64_t &lf = link_free_[(size_t)src * (G + 1) + G];
+    int64_t t0 = std::max(ready, lf);
+    int64_t t1 = t0 + dur(bytes, topo_.bw_at(src, G));
+    lf = t1;
+    Rec R;
+    std::memset(&R.r, 0, sizeof(R.r));
+    R.r.seq = seq_++;
+    R.r.kind = XK_REC_D2H;
+    R.r.operand = operand;
+    R.r.bi = e.bi;
+    R.r.bj = e.bj;
+    R.r.tk = -1;
+    R.r.version = e.ver;
+    R.r.dst = XK_HOST;
+    R.r.src = src;
+    R.r.src_state = XK_SRC_VALID;
+    R.r.depth = 0;
+    R.r.t_start = t0;
+    R.r.t_end = t1;
+    R.r.work = bytes;
+    R.r.dep[0] = dep;
+    R.r.dep[1] = R.r.dep[2] = R.r.dep[3] = -1;
+    R.key = key;
+    R.sub_r0 = r0;
+    R.sub_c0 = c0;
+    R.sub_rows = rows;
+    R.sub_cols = cols;
+    out.push_back(R);
+    if (r0 == 0 && c0 == 0 && rows == e.rows && cols == e.cols) {
+        e.host.present = true;
+        e.host.ver = e.ver;
+        e.host.t_done = t1;
+        e.host.producer = R.r.seq;
+        e.host.depth = 0;
+    }
+}
+
+// steps 2, 3, 6, 7: per-GPU k-major lists in k-shifted anti-diagonal order, event loop
+// on the smallest request time, task timing, output versioning, D2H after last writer.
+int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double beta, char ta,
+                       char tb, std::vector<Rec> &out, std::string &err) {
+    const int G = topo_.G;
+    const int W = std::max(1, flags_.window);
+    // pending reads per (key, version) in this call
+    std::map<std::pair<int, int64_t>, int64_t> readers;
+    for (auto &t : tasks)
+        for (auto &in : t.in) readers[{in.key, in.ver}]++;
+    std::vector<std::vector<int>> lists(G);
+    int64_t tmax = 1;
+    for (auto &t : tasks) tmax = std::max(tmax, std::max(t.i, t.j) + 1);
+    for (size_t q = 0; q < tasks.size(); ++q) lists[tasks[q].gpu].push_back((int)q);
+    for (int d = 0; d < G; ++d) {
+        std::stable_sort(lists[d].begin(), lists[d].end(), [&](int a, int b) {
+            const Task &x = tasks[a], &y = tasks[b];
+            int64_t kx = std::max<int64_t>(x.tk, 0), ky = std::max<int64_t>(y.tk, 0);
+            auto key = [&](const Task &t, int64_t k) {
+                return std::make_tuple(k, (t.i + t.j + k) % tmax, t.i, t.j);
+            };
+            return key(x, kx) < key(y, ky);
+        });
+    }
+    std::vector<size_t> pos(G, 0);
+    auto ready = [&](const Task &t) {
+        for (auto &in : t.in)
+            if (entries_[in.key].ver != in.ver) return false;
+        const Entry &o = entries_[t.out_key];
+        if (o.ver != t.out_ver - 1) return false;
+        auto it = readers.find({t.out_key, t.out_ver - 1});
+        int64_t pend = (it == readers.end()) ? 0 : it->second;
+        for (auto &in : t.in)
+            if (in.key == t.out_key && in.ver == t.out_ver - 1) pend--;
+        return pend == 0;
+    };
+    size_t done = 0;
+    while (done < tasks.size()) {
+        int best = -1;
+        int64_t best_treq = 0;
+        for (int d = 0; d < G; ++d) {
+            if (pos[d] == lists[d].size()) continue;
+            const Task &t = tasks[lists[d][pos[d]]];
+            if (!ready(t)) continue;
+            const auto &h = ends_[d];
+            int64_t treq = (int64_t)h.size() >= W ? h[h.size() - W] : 0;
+            if (best < 0 || treq < best_treq) { best = d; best_treq = treq; }
+        }
+        if (best < 0) {
+            err = "planner deadlock (no ready task)";
+            return XK_ERR_INTERNAL;
+        }
+        const int d = best;
+        Task &t = tasks[lists[d][pos[d]]];
+        const int64_t treq = best_treq;
+        int64_t in_ready = 0;
+        int64_t deps[4] = {-1, -1, -1, -1};
+        for (auto &in : t.in) {
+            Entry &e = entries_[in.key];
+            if (!(e.gpu[d].present && e.gpu[d].ver == in.ver) &&
+                !emit_copy(in.key, in.ver, d, treq, in.operand, out)) {
+                err = "no valid copy of an input tile (invalidated without coherence?)";
+                return XK_ERR_INTERNAL;
+            }
+            in_ready = std::max(in_ready, e.gpu[d].t_done);
+            deps[in.operand] = e.gpu[d].producer;
+            readers[{in.key, in.ver}]--;
+        }
+        int64_t t0 = std::max(gpu_free_[d], in_ready);
+        int64_t t1 = t0 + dur(t.flops, topo_.rate_mflops);
+        gpu_free_[d] = t1;
+        ends_[d].push_back(t1);
+        Entry &o = entries_[t.out_key];
+        Rec R;
+        std::memset(&R.r, 0, sizeof(R.r));
+        R.r.seq = seq_++;
+        R.r.kind = XK_REC_TASK;
+        R.r.operand = 2;
+        R.r.bi = o.bi;
+        R.r.bj = o.bj;
+        R.r.tk = t.tk;
+        R.r.version = t.out_ver;
+        R.r.dst = d;
+        R.r.src = d;
+        R.r.src_state = XK_SRC_NONE;
+        R.r.depth = 0;
+        R.r.t_start = t0;
+        R.r.t_end = t1;
+        R.r.work = t.flops;
+        for (int q = 0; q < 4; ++q) R.r.dep[q] = deps[q];
+        R.key = t.out_key;
+        R.keyA = t.keyA;
+        R.keyB = t.keyB;
+        R.ta = ta;
+        R.tb = tb;
+        R.alpha = alpha;
+        // beta applies on the first task of the chain only (k == 0 or scale-only)
+        R.beta = (t.tk <= 0) ? beta : 1.0;
+        R.m = t.m;
+        R.n = t.n;
+        R.k = t.k;
+        out.push_back(R);
+        o.ver = t.out_ver;
+        for (int g = 0; g < G; ++g)
+            if (g != d) o.gpu[g].present = false;
+        o.gpu[d].present = true;
+        o.gpu[d].ver = t.out_ver;
+        o.gpu[d].t_done = t1;
+        o.gpu[d].producer = R.r.seq;
+        o.gpu[d].depth = 0;
+        if (sync && t.last_writer)
+            emit_d2h(t.out_key, d, 0, 0, o.rows, o.cols, t1, R.r.seq, 2, out);
+        pos[d]++;
+        done++;
+    }
+    return XK_OK;
+}
+
+int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
+    const int64_t m = c.m, n = c.n, k = c.k, T = flags_.T;
+    const bool ta = c.transA == 'T' || c.transA == 't' || c.transA == 'C' || c.transA == 'c';
+    const bool tb = c.transB == 'T' || c.transB == 't' || c.transB == 'C' || c.transB == 'c';
+    if (m == 0 || n == 0 || ((c.alpha == 0.0 || k == 0) && c.beta == 1.0)) return XK_OK;
+    const bool scale_only = (c.alpha == 0.0 || k == 0);
+    int mc = find_or_add_matrix(c.C, (int64_t)c.ldc, m, n, err);
+    if (mc < 0) return XK_ERR_UNSUPPORTED;
+    int ma = -1, mb = -1;
+    if (!scale_only) {
+        ma = find_or_add_matrix(c.A, (int64_t)c.lda, ta ? k : m, ta ? m : k, err);
+        if (ma < 0) return XK_ERR_UNSUPPORTED;
+        mb = find_or_add_matrix(c.B, (int64_t)c.ldb, tb ? n : k, tb ? k : n, err);
+        if (mb < 0) return XK_ERR_UNSUPPORTED;
+    }
+    const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
+    std::vector<Task> tasks;
+    for (int64_t j = 0; j < tn; ++j) {
+        for (int64_t i = 0; i < tm; ++i) {
+            int keyC = key_of(mc, i, j);
+            int64_t v0 = entries_[keyC].ver;
+            int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
+            if (scale_only) {
+                Task t;
+                t.gpu = owner(i, j);
+                t.out_key = keyC;
+                t.out_ver = v0 + 1;
+                if (c.beta != 0.0) t.in.push_back({keyC, v0, 2});
+                t.tk = -1;
+                t.i = i; t.j = j;
+                t.m = mt; t.n = nt; t.k = 0;
+                t.flops = mt * nt;
+                t.last_writer = true;
+                tasks.push_back(t);
+                continue;
+            }
+            for (int64_t kk = 0; kk < tkn; ++kk) {
+                int64_t kt = std::min(T, k - kk * T);
+                int keyA = ta ? key_of(ma, kk, i) : key_of(ma, i, kk);
+                int keyB = tb ? key_of(mb, j, kk) : key_of(mb, kk, j);
+                Task t;
+                t.gpu = owner(i, j);
+                t.out_key = keyC;
+                t.out_ver = v0 + kk + 1;
+                t.in.push_back({keyA, entries_[keyA].ver, 0});
+                t.in.push_back({keyB, entries_[keyB].ver, 1});
+                if (kk > 0) t.in.push_back({keyC, v0 + kk, 2});
+                else if (c.beta != 0.0) t.in.push_back({keyC, v0, 2});
+                t.tk = kk;
+                t.i = i; t.j = j;
+                t.m = mt; t.n = nt; t.k = kt;
+                t.flops = 2 * mt * nt * kt;
+                t.last_writer = (kk == tkn - 1);
+                t.keyA = keyA;
+                t.keyB = keyB;
+                tasks.push_back(t);
+            }
+        }
+    }
+    return run_tasks(tasks, c.sync != 0, c.alpha, c.beta, ta ? 'T' : 'N', tb ? 'T' : 'N', out, err);
+}
+
+bool Planner::view_tiles(uint64_t base, int64_t m, int64_t n, int64_t ld, int *mat, int64_t *r0,
+                         int64_t *c0) const {
+    for (size_t i = 0; i < mats_.size(); ++i) {
+        const Matrix &M = mats_[i];
+        if (M.ld != ld || M.ld < 0) continue;
+        if (base < M.base) continue;
+        uint64_t off = (base - M.base) / 8;
+        int64_t rr = (int64_t)(off % (uint64_t)ld), cc = (int64_t)(off / (uint64_t)ld);
+        if (rr < M.rows && cc < M.cols) {
+            *mat = (int)i;
+            *r0 = rr;
+            *c0 = cc;
+            (void)m; (void)n;
+            return true;
+        }
+    }
+    return false;
+}
+
+// step 10: partial coherence writes back only the stale tile intersections;
+// prefetch (data-on-device) loads tiles onto their owner GPUs.
+int Planner::plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::string &err,
+                           bool prefetch) {
+    const int64_t T = flags_.T;
+    if (c.m <= 0 || c.n <= 0) return XK_OK;
+    int mat;
+    int64_t r0, c0;
+    if (prefetch) {
+        mat = find_or_add_matrix(c.C, (int64_t)c.ldc, c.m, c.n, err);
+        if (mat < 0) return XK_ERR_UNSUPPORTED;
+        for (int64_t bj = 0; bj < cdiv(c.n, T); ++bj)
+            for (int64_t bi = 0; bi < cdiv(c.m, T); ++bi) {
+                int key = key_of(mat, bi, bj);
+                Entry &e = entries_[key];
+                int d = owner(bi, bj);
+                if (e.gpu[d].present && e.gpu[d].ver == e.ver) continue;
+                if (!emit_copy(key, e.ver, d, 0, 2, out)) {
+                    err = "prefetch: no valid copy of a tile";
+                    return XK_ERR_INTERNAL;
+                }
+            }
+        return XK_OK;
+    }
+    if (!view_tiles(c.C, c.m, c.n, (int64_t)c.ldc, &mat, &r0, &c0)) return XK_OK;  // never cached
+    const Matrix &M = mats_[mat];
+    int64_t rend = std::min(M.rows, r0 + c.m), cend = std::min(M.cols, c0 + c.n);
+    for (int64_t bj = c0 / T; bj * T < cend; ++bj) {
+        for (int64_t bi = r0 / T; bi * T < rend; ++bi) {
+            std::string k(sizeof(int) + 2 * sizeof(int64_t), '\0');
+            std::memcpy(&k[0], &mat, sizeof(int));
+            std::memcpy(&k[sizeof(int)], &bi, sizeof(int64_t));
+            std::memcpy(&k[sizeof(int) + sizeof(int64_t)], &bj, sizeof(int64_t));
+            auto it = keymap_.find(k);
+            if (it == keymap_.end()) continue;
+            Entry &e = entries_[it->second];
+            if (e.host.present && e.host.ver == e.ver) continue;  // host already valid
+            int src = -1;
+            for (int g = 0; g < topo_.G; ++g) {
+                const NodeCopy &cp = e.gpu[g];
+                if (!cp.present || cp.ver != e.ver) continue;
+                if (src < 0 || cp.t_done < e.gpu[src].t_done) src = g;
+            }
+            if (src < 0) {
+                err = "coherence: no valid copy of a stale tile";
+                return XK_ERR_INTERNAL;
+            }
+            int64_t tr0 = std::max(r0, bi * T) - bi * T, tc0 = std::max(c0, bj * T) - bj * T;
+            int64_t tr1 = std::min(rend, bi * T + e.rows) - bi * T;
+            int64_t tc1 = std::min(cend, bj * T + e.cols) - bj * T;
+            if (tr1 <= tr0 || tc1 <= tc0) continue;
+            emit_d2h(it->second, src, tr0, tc0, tr1 - tr0, tc1 - tc0, e.gpu[src].t_done,
+                     e.gpu[src].producer, 2, out);
+        }
+    }
+    return XK_OK;
+}
+
+void Planner::full_sync() {
+    for (auto &e : entries_) {
+        e.host.t_done = 0;
+        e.host.producer = -1;
+        for (auto &g : e.gpu) {
+            g.t_done = 0;
+            g.producer = -1;
+        }
+    }
+    std::fill(link_free_.begin(), link_free_.end(), 0);
+    std::fill(gpu_free_.begin(), gpu_free_.end(), 0);
+    for (auto &h : ends_) h.clear();
+}
+
+void Planner::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
+    int mat;
+    int64_t r0, c0;
+    if (m <= 0 || n <= 0) return;
+    if (!view_tiles(base, m, n, ld, &mat, &r0, &c0)) return;
+    const int64_t T = flags_.T;
+    const Matrix &M = mats_[mat];
+    int64_t rend = std::min(M.rows, r0 + m), cend = std::min(M.cols, c0 + n);
+    for (auto &kv : keymap_) {
+        Entry &e = entries_[kv.second];
+        if (e.mat != mat) continue;
+        if (e.bi * T >= rend || e.bi * T + e.rows <= r0) continue;
+        if (e.bj * T >= cend || e.bj * T + e.cols <= c0) continue;
+        for (auto &g : e.gpu) g.present = false;
+    }
+}
+
+int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
+    switch (c.routine) {
+    case XK_ROUTINE_DGEMM: {
+        int rc = plan_gemm(c, out, err);
+        if (rc) return rc;
+        if (c.sync) {
+            // the library waits here; then a full sync point and invalidation of the
+            // operands' device copies (sync routines are drop-in)
+            full_sync();
+            const bool ta = c.transA == 'T' || c.transA == 't' || c.transA == 'C' || c.transA == 'c';
+            const bool tb = c.transB == 'T' || c.transB == 't' || c.transB == 'C' || c.transB == 'c';
+            if (c.alpha != 0.0 && c.k > 0) {
+                invalidate(c.A, ta ? c.k : c.m, ta ? c.m : c.k, (int64_t)c.lda);
+                invalidate(c.B, tb ? c.n : c.k, tb ? c.k : c.n, (int64_t)c.ldb);
+            }
+            invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        }
+        return XK_OK;
+    }
+    case XK_ROUTINE_COHERENT:
+        return plan_coherent(c, out, err, false);
+    case XK_ROUTINE_SYNC:
+        full_sync();
+        return XK_OK;
+    case XK_ROUTINE_INVALIDATE:
+        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        return XK_OK;
+    case XK_ROUTINE_PREFETCH:
+        return plan_coherent(c, out, err, true);
+    default:
+        err = "unknown routine";
+        return XK_ERR_CONFIG;
+    }
+}
+
+}  // namespace xk

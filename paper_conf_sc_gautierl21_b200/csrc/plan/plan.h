@@ -1,0 +1,139 @@
+// plan.h -- the XKBlas planner: tiling, owner-computes map, coherence directory,
+// source selection (topology-aware + optimistic forwarding) and the deterministic
+// integer virtual-time model that orders copies and tasks.  Pure C++ (no CUDA): the
+// same object drives the executor inside libxk.so and xk_plan_dump() for CPU tests.
+//
+// Paper: directory of tile copies P:408-412; "initiates data transfers of the tile from
+// one of the resources handling a valid copy once the scheduler has decided to map a
+// task" P:440-442; topology-aware order P:446-451; optimistic in-flight source
+// P:491-498; owner-computes P:384-389 on a 2D block-cyclic grid P:743-747.
+// Readings are listed in DESIGN.md.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "xk.h"
+
+namespace xk {
+
+struct Topology {
+    int G = 1;
+    std::vector<int64_t> bw;  // (G+1)^2 MB/s, row = src, col = dst, index G = host
+    int64_t rate_mflops = 35000000;
+    int64_t bw_at(int s, int d) const { return bw[(size_t)s * (G + 1) + d]; }
+};
+
+struct Flags {
+    int topo = XK_TOPO_RANKED;
+    int optimistic = 1;
+    int window = 2;
+    int P = 1, Q = 1;
+    int64_t T = 2048;
+};
+
+// A host matrix as the planner sees it: identity (base, ld) and stored extent.
+struct Matrix {
+    uint64_t base = 0;
+    int64_t ld = 0;
+    int64_t rows = 0, cols = 0;  // stored extent covered by the tiles known so far
+};
+
+struct NodeCopy {
+    bool present = false;
+    int64_t ver = 0;
+    int64_t t_done = 0;    // virtual time the copy is complete
+    int64_t producer = -1; // seq of the record that produced it (-1 = complete/original)
+    int depth = 0;
+};
+
+struct Entry {
+    int mat = -1;
+    int64_t bi = 0, bj = 0;
+    int64_t rows = 0, cols = 0;  // tile extent (ragged at the edges)
+    int64_t ver = 0;             // current (latest planned) version
+    NodeCopy host;               // host copy (present & ver == cur -> host valid)
+    std::vector<NodeCopy> gpu;   // per GPU
+};
+
+// A plan record plus what the executor needs to act on it.
+struct Rec {
+    xk_plan_rec_t r;
+    int key = -1;                 // directory entry id
+    int64_t sub_r0 = 0, sub_c0 = 0, sub_rows = 0, sub_cols = 0;  // D2H intersection (tile-relative)
+    // task description (TASK records)
+    char ta = 'N', tb = 'N';
+    double alpha = 1.0, beta = 0.0;
+    int keyA = -1, keyB = -1;     // input tiles on dst (-1: none)
+    int64_t m = 0, n = 0, k = 0;  // task shape
+};
+
+class Planner {
+public:
+    Planner(const Topology &t, const Flags &f);
+
+    // Plan one call; appends records to out.  Returns 0 or XK_ERR_*.
+    int plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
+
+    // Full synchronisation point (return of a sync routine, xk_sync): every copy is
+    // complete, clocks restart at 0.
+    void full_sync();
+    // Drop GPU copies of the tiles intersecting a view.
+    void invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld);
+
+    const Entry &entry(int id) const { return entries_[id]; }
+    const Matrix &matrix(int id) const { return mats_[id]; }
+    int G() const { return topo_.G; }
+    int owner(int64_t i, int64_t j) const {
+        return (int)((i % flags_.P) * flags_.Q + (j % flags_.Q));
+    }
+    const Flags &flags() const { return flags_; }
+    int link_class(int s, int d) const { return cls_[(size_t)s * (topo_.G + 1) + d]; }
+
+private:
+    struct Input { int key; int64_t ver; int operand; };
+    struct Task {
+        int gpu;
+        int out_key;
+        int64_t out_ver;            // version produced
+        std::vector<Input> in;      // in operand order A, B, C
+        int64_t tk;                 // k index, -1 scale-only
+        int64_t i, j;               // output tile coords (op space)
+        int64_t m, n, k;            // shape
+        int64_t flops;
+        bool last_writer;           // last write of out_key in this call
+        int keyA = -1, keyB = -1;
+    };
+
+    int find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t cols, std::string &err);
+    int key_of(int mat, int64_t bi, int64_t bj);
+    int64_t dur(int64_t amount, int64_t rate) const;  // ceil(amount*1000/rate) ns
+    int select_source(const Entry &e, int64_t ver, int d, int64_t treq, int *state) const;
+    bool emit_copy(int key, int64_t ver, int d, int64_t treq, int operand, std::vector<Rec> &out);
+    void emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, int64_t cols,
+                  int64_t ready, int64_t dep, int operand, std::vector<Rec> &out);
+    int plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
+    int plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::string &err, bool prefetch);
+    int run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double beta, char ta,
+                  char tb, std::vector<Rec> &out, std::string &err);
+    bool view_tiles(uint64_t base, int64_t m, int64_t n, int64_t ld, int *mat,
+                    int64_t *r0, int64_t *c0) const;
+
+    Topology topo_;
+    Flags flags_;
+    std::vector<int> cls_;
+    std::vector<Matrix> mats_;
+    std::vector<Entry> entries_;
+    std::unordered_map<std::string, int> keymap_;
+    std::vector<int64_t> link_free_;     // (G+1)^2
+    std::vector<int64_t> gpu_free_;      // G
+    std::vector<std::vector<int64_t>> ends_;  // per GPU task end-time history (since last sync)
+    int64_t seq_ = 0;
+};
+
+// Link classes: distinct off-diagonal bandwidths sorted
+// ascending, new class when consecutive values differ by a ratio > 1.25.
+std::vector<int> link_classes(int G, const std::vector<int64_t> &bw);
+
+}  // namespace xk
