@@ -328,7 +328,7 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double
             if (best < 0 || treq < best_treq) { best = d; best_treq = treq; }
         }
         if (best < 0) {
-            err = "planner deadlock (no ready task)";
+            err = "planner deadlock: no ready task (output aliases an input?)";
             return XK_ERR_INTERNAL;
         }
         const int d = best;

@@ -15,7 +15,8 @@ def pytest_configure(config):
 
 @pytest.fixture(scope="session", autouse=True)
 def _native_builds():
-    from tools.build_native import build_inputs, build_oracle
+    from tools.build_native import build_inputs, build_oracle, build_xk
     build_inputs()
     build_oracle()
+    build_xk()
     yield
