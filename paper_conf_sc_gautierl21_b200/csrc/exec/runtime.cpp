@@ -1,0 +1,718 @@
+// runtime.cpp -- executor of plan records (see runtime.h).
+//
+// Ordering is enforced with CUDA events, never by the virtual-time model: every record
+// waits on the events of the records it depends on (plan deps = RAW), and a buffer that is
+// overwritten first waits on the reads of its previous contents (WAR) and its previous
+// write (WAW).  Records are issued by one host thread in plan order, and every dependency
+// names an earlier record, so no cudaStreamWaitEvent is ever issued before the matching
+// cudaEventRecord (the issue-order hazard of SURVEY.md §0.1).
+#include "exec/runtime.h"
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstdio>
+#include <cstring>
+
+#include "api/common.h"
+#include "kernels/kernels.h"
+
+namespace xk {
+
+#define XK_CK(call)                                        \
+    do {                                                   \
+        cudaError_t _e = (call);                           \
+        if (_e != cudaSuccess) return cuda_fail(_e, #call); \
+    } while (0)
+
+static inline int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
+
+int Runtime::cuda_fail(cudaError_t e, const char *what) {
+    set_error(std::string(what) + ": " + cudaGetErrorString(e));
+    return XK_ERR_CUDA;
+}
+
+int Runtime::set_dev(int g) {
+    int p = devs_[g].phys;
+    if (p != cur_dev_) {
+        XK_CK(cudaSetDevice(p));
+        cur_dev_ = p;
+    }
+    return XK_OK;
+}
+
+Runtime::~Runtime() {}
+
+int Runtime::init(const xk_config_t &cfg) {
+    cfg_ = cfg;
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) {
+        set_error(std::string("no CUDA device: ") + cudaGetErrorString(e));
+        return XK_ERR_NO_DEVICE;
+    }
+    int G = cfg.ngpus > 0 ? cfg.ngpus : ndev;
+    if (G > XK_MAX_GPUS) {
+        set_error("ngpus > XK_MAX_GPUS");
+        return XK_ERR_CONFIG;
+    }
+    devs_.assign(G, Device());
+    for (int g = 0; g < G; ++g) {
+        int p = cfg.map_devices ? cfg.phys[g] : g % ndev;
+        if (p < 0 || p >= ndev) {
+            set_error("logical->physical device map out of range");
+            return XK_ERR_CONFIG;
+        }
+        devs_[g].phys = p;
+    }
+    int ks = cfg.kstreams > 0 ? std::min(cfg.kstreams, kMaxKStreams) : 2;
+    cfg_.kstreams = ks;
+    // peer access between distinct physical devices (NVLink / NVSwitch)
+    for (int a = 0; a < G; ++a)
+        for (int b = 0; b < G; ++b) {
+            int pa = devs_[a].phys, pb = devs_[b].phys;
+            if (pa == pb) continue;
+            int can = 0;
+            XK_CK(cudaDeviceCanAccessPeer(&can, pa, pb));
+            if (!can) continue;
+            XK_CK(cudaSetDevice(pa));
+            cudaError_t pe = cudaDeviceEnablePeerAccess(pb, 0);
+            if (pe != cudaSuccess && pe != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(pe, "cudaDeviceEnablePeerAccess");
+            cudaGetLastError();
+        }
+    for (int g = 0; g < G; ++g) {
+        Device &d = devs_[g];
+        XK_CK(cudaSetDevice(d.phys));
+        XK_CK(cudaStreamCreateWithFlags(&d.h2d, cudaStreamNonBlocking));
+        XK_CK(cudaStreamCreateWithFlags(&d.d2h, cudaStreamNonBlocking));
+        XK_CK(cudaStreamCreateWithFlags(&d.p2p, cudaStreamNonBlocking));
+        for (int k = 0; k < ks; ++k) XK_CK(cudaStreamCreateWithFlags(&d.ks[k], cudaStreamNonBlocking));
+    }
+    cur_dev_ = -1;
+    ev_pool_.assign(G, {});
+    ev_used_.assign(G, {});
+    // flags
+    flags_.topo = cfg.topo;
+    flags_.optimistic = cfg.optimistic;
+    flags_.window = cfg.window > 0 ? cfg.window : 2;
+    flags_.T = cfg.tile > 0 ? cfg.tile : 2048;
+    flags_.P = cfg.grid_p;
+    flags_.Q = cfg.grid_q;
+    if (flags_.P <= 0 || flags_.Q <= 0) default_grid(G, &flags_.P, &flags_.Q);
+    if (flags_.P * flags_.Q != G || flags_.topo < 0 || flags_.topo > 2) {
+        set_error("config: grid P*Q must equal ngpus; topo in {0,1,2}");
+        return XK_ERR_CONFIG;
+    }
+    // topology (a1): defaults, then the measured matrix when probing
+    topo.G = G;
+    topo.bw.assign((size_t)(G + 1) * (G + 1), 0);
+    for (int s = 0; s <= G; ++s)
+        for (int d = 0; d <= G; ++d) {
+            int64_t v;
+            if (s == G || d == G) v = (s == d) ? 3000000 : 55000;
+            else if (s == d) v = 3000000;
+            else v = (devs_[s].phys == devs_[d].phys) ? 1500000 : 700000;
+            topo.bw[(size_t)s * (G + 1) + d] = v;
+        }
+    topo.rate_mflops = cfg.task_rate_mflops > 0 ? cfg.task_rate_mflops : 35000000;
+    perf_rank.assign((size_t)G * G, 0);
+    for (int s = 0; s < G; ++s)
+        for (int d = 0; d < G; ++d) {
+            int ps = devs_[s].phys, pd = devs_[d].phys;
+            if (ps == pd) continue;
+            int v = 0;
+            if (cudaDeviceGetP2PAttribute(&v, cudaDevP2PAttrPerformanceRank, ps, pd) == cudaSuccess)
+                perf_rank[(size_t)s * G + d] = v;
+            cudaGetLastError();
+        }
+    if (cfg.probe) {
+        int rc = probe_topology();
+        if (rc) return rc;
+    }
+    planner_.reset(new Planner(topo, flags_));
+    std::memset(&stats, 0, sizeof(stats));
+    stats.ngpus = G;
+    return XK_OK;
+}
+
+// a1: time pinned H2D/D2H per GPU and CE copies for every ordered GPU pair; the FP64
+// tile rate from one T x T x T tile GEMM.  Untimed by the API ("store the
+// performance of link during the library initialization").
+int Runtime::probe_topology() {
+    const int G = (int)devs_.size();
+    const size_t bytes = (size_t)64 << 20;
+    void *host = nullptr;
+    XK_CK(cudaMallocHost(&host, bytes));
+    std::memset(host, 1, bytes);
+    std::vector<void *> dbuf(G, nullptr), dbuf2(G, nullptr);
+    for (int g = 0; g < G; ++g) {
+        XK_CK(cudaSetDevice(devs_[g].phys));
+        XK_CK(cudaMalloc(&dbuf[g], bytes));
+        XK_CK(cudaMalloc(&dbuf2[g], bytes));
+    }
+    auto timed = [&](int g, cudaStream_t s, auto fn, float *ms_out) -> int {
+        XK_CK(cudaSetDevice(devs_[g].phys));
+        cudaEvent_t a, b;
+        XK_CK(cudaEventCreate(&a));
+        XK_CK(cudaEventCreate(&b));
+        float best = 1e30f;
+        for (int rep = 0; rep < 3; ++rep) {
+            XK_CK(cudaEventRecord(a, s));
+            XK_CK(fn());
+            XK_CK(cudaEventRecord(b, s));
+            XK_CK(cudaEventSynchronize(b));
+            float ms = 0;
+            XK_CK(cudaEventElapsedTime(&ms, a, b));
+            if (rep > 0) best = std::min(best, ms);
+        }
+        cudaEventDestroy(a);
+        cudaEventDestroy(b);
+        *ms_out = best;
+        return XK_OK;
+    };
+    auto mbps = [&](float ms) { return (int64_t)((double)bytes / (ms * 1e-3) / 1e6); };
+    const int N = G + 1;
+    for (int g = 0; g < G; ++g) {
+        float ms;
+        int rc = timed(g, devs_[g].h2d, [&] { return cudaMemcpyAsync(dbuf[g], host, bytes, cudaMemcpyHostToDevice, devs_[g].h2d); }, &ms);
+        if (rc) return rc;
+        topo.bw[(size_t)G * N + g] = mbps(ms);
+        rc = timed(g, devs_[g].d2h, [&] { return cudaMemcpyAsync(host, dbuf[g], bytes, cudaMemcpyDeviceToHost, devs_[g].d2h); }, &ms);
+        if (rc) return rc;
+        topo.bw[(size_t)g * N + G] = mbps(ms);
+        rc = timed(g, devs_[g].p2p, [&] { return cudaMemcpyAsync(dbuf2[g], dbuf[g], bytes, cudaMemcpyDeviceToDevice, devs_[g].p2p); }, &ms);
+        if (rc) return rc;
+        topo.bw[(size_t)g * N + g] = mbps(ms);
+    }
+    for (int s = 0; s < G; ++s)
+        for (int d = 0; d < G; ++d) {
+            if (s == d) continue;
+            float ms;
+            int rc = timed(d, devs_[d].p2p, [&] { return cudaMemcpyAsync(dbuf[d], dbuf[s], bytes, cudaMemcpyDeviceToDevice, devs_[d].p2p); }, &ms);
+            if (rc) return rc;
+            topo.bw[(size_t)s * N + d] = mbps(ms);
+        }
+    topo.bw[(size_t)G * N + G] = topo.bw[0];
+    // FP64 tile-task rate on GPU 0 (one T x T x T tile GEMM, T <= 2048)
+    if (cfg_.task_rate_mflops <= 0) {
+        int64_t T = std::min<int64_t>(flags_.T, 2048);
+        size_t tb = (size_t)T * T * 8;
+        double *a = nullptr, *b = nullptr, *c = nullptr;
+        XK_CK(cudaSetDevice(devs_[0].phys));
+        XK_CK(cudaMalloc(&a, tb));
+        XK_CK(cudaMalloc(&b, tb));
+        XK_CK(cudaMalloc(&c, tb));
+        XK_CK(cudaMemsetAsync(a, 0, tb, devs_[0].ks[0]));
+        XK_CK(cudaMemsetAsync(b, 0, tb, devs_[0].ks[0]));
+        XK_CK(cudaMemsetAsync(c, 0, tb, devs_[0].ks[0]));
+        float ms;
+        int rc = timed(0, devs_[0].ks[0], [&] { return launch_dgemm_tile(false, false, T, T, T, 1.0, a, T, b, T, 1.0, c, T, devs_[0].ks[0]); }, &ms);
+        cudaFree(a);
+        cudaFree(b);
+        cudaFree(c);
+        if (rc) return rc;
+        topo.rate_mflops = std::max<int64_t>(1, (int64_t)(2.0 * T * T * T / (ms * 1e3)));
+    }
+    for (int g = 0; g < G; ++g) {
+        cudaSetDevice(devs_[g].phys);
+        cudaFree(dbuf[g]);
+        cudaFree(dbuf2[g]);
+    }
+    cudaFreeHost(host);
+    cur_dev_ = -1;
+    return XK_OK;
+}
+
+cudaEvent_t Runtime::new_event(int g) {
+    auto &pool = ev_pool_[g];
+    cudaEvent_t e = nullptr;
+    if (!pool.empty()) {
+        e = pool.back();
+        pool.pop_back();
+    } else if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
+        return nullptr;
+    }
+    ev_used_[g].push_back(e);
+    return e;
+}
+
+int Runtime::record(cudaStream_t s, int g, Ev *out) {
+    cudaEvent_t e = new_event(g);
+    if (!e) return cuda_fail(cudaGetLastError(), "cudaEventCreate");
+    XK_CK(cudaEventRecord(e, s));
+    out->e = e;
+    out->s = s;
+    return XK_OK;
+}
+
+int Runtime::wait_on(cudaStream_t s, const Ev &ev) {
+    if (!ev.e || ev.s == s) return XK_OK;  // same stream: already ordered
+    XK_CK(cudaStreamWaitEvent(s, ev.e, 0));
+    return XK_OK;
+}
+
+int Runtime::wait_dep(cudaStream_t s, int64_t seq) {
+    if (seq < 0) return XK_OK;
+    auto it = seq_ev_.find(seq);
+    if (it == seq_ev_.end()) return XK_OK;  // completed before the last full sync
+    return wait_on(s, it->second);
+}
+
+static void add_reader(Buffer &b, const Ev &ev) {
+    for (auto &r : b.readers)
+        if (r.s == ev.s) {  // in-order stream: the newer event subsumes the older one
+            r = ev;
+            return;
+        }
+    b.readers.push_back(ev);
+}
+
+double *Runtime::alloc(int g, size_t bytes, int *rc) {
+    Device &d = devs_[g];
+    auto it = d.free_bufs.find(bytes);
+    if (it != d.free_bufs.end() && !it->second.empty()) {
+        double *p = it->second.back();
+        it->second.pop_back();
+        d.bytes_in_use += bytes;
+        return p;
+    }
+    if ((*rc = set_dev(g))) return nullptr;
+    double *p = nullptr;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        // give cached free buffers of this device back and retry once
+        for (auto &kv : d.free_bufs)
+            for (double *q : kv.second) {
+                cudaFree(q);
+                for (auto a = d.all_bufs.begin(); a != d.all_bufs.end(); ++a)
+                    if (a->first == q) { d.all_bufs.erase(a); break; }
+            }
+        d.free_bufs.clear();
+        e = cudaMalloc(&p, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            set_error("device tile cache full (no eviction): cudaMalloc failed");
+            *rc = XK_ERR_OOM;
+            return nullptr;
+        }
+    }
+    d.all_bufs.push_back({p, bytes});
+    d.bytes_in_use += bytes;
+    return p;
+}
+
+void Runtime::free_buf(int g, double *p, size_t bytes) {
+    devs_[g].free_bufs[bytes].push_back(p);
+    devs_[g].bytes_in_use -= bytes;
+}
+
+Buffer *Runtime::buf(int key, int g, bool create, int *rc) {
+    int64_t id = (int64_t)key * XK_MAX_GPUS + g;
+    auto it = bufs_.find(id);
+    if (it != bufs_.end()) return &it->second;
+    if (!create) {
+        set_error("internal: missing device tile");
+        *rc = XK_ERR_INTERNAL;
+        return nullptr;
+    }
+    const Entry &e = planner_->entry(key);
+    Buffer b;
+    b.ld = round_up(e.rows, 16);
+    b.bytes = (size_t)b.ld * e.cols * 8;
+    b.p = alloc(g, b.bytes, rc);
+    if (!b.p) return nullptr;
+    return &(bufs_[id] = b);
+}
+
+int Runtime::issue(const Rec &R) {
+    const xk_plan_rec_t &r = R.r;
+    const Entry &e = planner_->entry(R.key);
+    const Matrix &M = planner_->matrix(e.mat);
+    const int64_t T = flags_.T;
+    int rc = XK_OK;
+    switch (r.kind) {
+    case XK_REC_H2D: {
+        const int g = r.dst;
+        if ((rc = set_dev(g))) return rc;
+        Buffer *B = buf(R.key, g, true, &rc);
+        if (!B) return rc;
+        cudaStream_t s = devs_[g].h2d;
+        if ((rc = wait_dep(s, r.dep[0]))) return rc;
+        for (auto &rd : B->readers)
+            if ((rc = wait_on(s, rd))) return rc;
+        if ((rc = wait_on(s, B->writer))) return rc;
+        const char *host = (const char *)(uintptr_t)M.base + (e.bi * T + e.bj * T * M.ld) * 8;
+        if ((rc = copy_host(true, B->p, B->ld, (char *)host, M.ld, e.rows, e.cols, s))) return rc;
+        Ev ev;
+        if ((rc = record(s, g, &ev))) return rc;
+        seq_ev_[r.seq] = ev;
+        B->writer = ev;
+        B->readers.clear();
+        stats.h2d_bytes[g] += r.work;
+        return XK_OK;
+    }
+    case XK_REC_P2P: {
+        const int g = r.dst, gs = r.src;
+        Buffer *S = buf(R.key, gs, false, &rc);
+        if (!S) return rc;
+        if ((rc = set_dev(g))) return rc;
+        Buffer *D = buf(R.key, g, true, &rc);
+        if (!D) return rc;
+        S = buf(R.key, gs, false, &rc);  // rehash may have moved it
+        cudaStream_t s = devs_[g].p2p;
+        if ((rc = wait_dep(s, r.dep[0]))) return rc;
+        if ((rc = wait_on(s, S->writer))) return rc;
+        for (auto &rd : D->readers)
+            if ((rc = wait_on(s, rd))) return rc;
+        if ((rc = wait_on(s, D->writer))) return rc;
+        // store-and-forward of a whole compact tile over NVLink (copy engine, SMs stay free)
+        XK_CK(cudaMemcpyAsync(D->p, S->p, S->bytes, cudaMemcpyDeviceToDevice, s));
+        Ev ev;
+        if ((rc = record(s, g, &ev))) return rc;
+        seq_ev_[r.seq] = ev;
+        D->writer = ev;
+        D->readers.clear();
+        add_reader(*S, ev);
+        stats.p2p_in_bytes[g] += r.work;
+        stats.p2p_out_bytes[gs] += r.work;
+        if (r.src_state == XK_SRC_INFLIGHT) stats.forwards_inflight++;
+        else stats.forwards_valid++;
+        return XK_OK;
+    }
+    case XK_REC_TASK: {
+        const int g = r.dst;
+        if ((rc = set_dev(g))) return rc;
+        Buffer *O = buf(R.key, g, true, &rc);
+        if (!O) return rc;
+        Buffer *A = nullptr, *B = nullptr;
+        if (R.keyA >= 0) {
+            if (!(A = buf(R.keyA, g, false, &rc))) return rc;
+            if (!(B = buf(R.keyB, g, false, &rc))) return rc;
+            O = buf(R.key, g, false, &rc);
+        }
+        const Device &d = devs_[g];
+        uint64_t h = (uint64_t)(e.bi * 7919 + e.bj * 104729);
+        cudaStream_t s = d.ks[h % (uint64_t)cfg_.kstreams];
+        for (int q = 0; q < 4; ++q)
+            if ((rc = wait_dep(s, r.dep[q]))) return rc;
+        for (auto &rd : O->readers)
+            if ((rc = wait_on(s, rd))) return rc;
+        if ((rc = wait_on(s, O->writer))) return rc;
+        cudaEvent_t t0 = nullptr, t1 = nullptr;
+        if (kernel_timing) {
+            XK_CK(cudaEventCreate(&t0));
+            XK_CK(cudaEventCreate(&t1));
+            XK_CK(cudaEventRecord(t0, s));
+        }
+        cudaError_t ke;
+        if (A) {
+            ke = launch_dgemm_tile(R.ta == 'T', R.tb == 'T', R.m, R.n, R.k, R.alpha, A->p, A->ld,
+                                   B->p, B->ld, R.beta, O->p, O->ld, s);
+        } else {
+            ke = launch_scale_tile(R.m, R.n, R.beta, O->p, O->ld, s);
+        }
+        if (ke != cudaSuccess) return cuda_fail(ke, "tile kernel launch");
+        if (kernel_timing) {
+            XK_CK(cudaEventRecord(t1, s));
+            ktimers_.push_back({t0, t1});
+        }
+        Ev ev;
+        if ((rc = record(s, g, &ev))) return rc;
+        seq_ev_[r.seq] = ev;
+        O->writer = ev;
+        O->readers.clear();
+        if (A) {
+            add_reader(*A, ev);
+            add_reader(*B, ev);
+        }
+        stats.tasks[g]++;
+        stats.flops[g] += r.work;
+        stats.kernel_launches++;
+        return XK_OK;
+    }
+    case XK_REC_D2H: {
+        const int gs = r.src;
+        if ((rc = set_dev(gs))) return rc;
+        Buffer *S = buf(R.key, gs, false, &rc);
+        if (!S) return rc;
+        cudaStream_t s = devs_[gs].d2h;
+        if ((rc = wait_dep(s, r.dep[0]))) return rc;
+        if ((rc = wait_on(s, S->writer))) return rc;
+        char *host = (char *)(uintptr_t)M.base +
+                     ((e.bi * T + R.sub_r0) + (e.bj * T + R.sub_c0) * M.ld) * 8;
+        const double *src = S->p + R.sub_r0 + R.sub_c0 * S->ld;
+        if ((rc = copy_host(false, (double *)src, S->ld, host, M.ld, R.sub_rows, R.sub_cols, s))) return rc;
+        Ev ev;
+        if ((rc = record(s, gs, &ev))) return rc;
+        seq_ev_[r.seq] = ev;
+        add_reader(*S, ev);
+        pending_d2h_.push_back(ev);
+        stats.d2h_bytes[gs] += r.work;
+        return XK_OK;
+    }
+    default:
+        set_error("internal: unknown record kind");
+        return XK_ERR_INTERNAL;
+    }
+}
+
+// Boundaries of host registrations strictly inside [lo, hi): a pinned copy must not
+// straddle two registrations (the driver rejects it), so copy_host splits there.
+std::vector<uintptr_t> Runtime::reg_cuts(uintptr_t lo, uintptr_t hi) const {
+    const uintptr_t page = 4096;
+    std::vector<uintptr_t> cuts;
+    auto scan = [&](const std::map<uintptr_t, size_t> &m) {
+        for (auto &kv : m) {
+            uintptr_t a = kv.first / page * page, b = (kv.first + kv.second + page - 1) / page * page;
+            if (lo < a && a < hi) cuts.push_back(a);
+            if (lo < b && b < hi) cuts.push_back(b);
+        }
+    };
+    scan(internal_reg_);
+    scan(registered_);
+    std::sort(cuts.begin(), cuts.end());
+    cuts.erase(std::unique(cuts.begin(), cuts.end()), cuts.end());
+    return cuts;
+}
+
+// 2D copy between a device tile (ld = dld) and a host view (ld = hld), split so that no
+// single copy crosses a host registration boundary.
+int Runtime::copy_host(bool h2d, double *dev, int64_t dld, char *host, int64_t hld, int64_t rows,
+                       int64_t cols, cudaStream_t s) {
+    const cudaMemcpyKind kind = h2d ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToHost;
+    const uintptr_t lo = (uintptr_t)host;
+    const uintptr_t hi = lo + (uintptr_t)(((cols - 1) * hld + rows) * 8);
+    std::vector<uintptr_t> cuts = reg_cuts(lo, hi);
+    auto cp2d = [&](int64_t c0, int64_t ncol) -> int {
+        char *h = host + c0 * hld * 8;
+        double *d = dev + c0 * dld;
+        cudaError_t e = h2d ? cudaMemcpy2DAsync(d, dld * 8, h, hld * 8, rows * 8, ncol, kind, s)
+                            : cudaMemcpy2DAsync(h, hld * 8, d, dld * 8, rows * 8, ncol, kind, s);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy2DAsync (tile)");
+        return XK_OK;
+    };
+    if (cuts.empty()) return cp2d(0, cols);
+    auto segment = [&](uintptr_t a) {  // index of the registration segment holding address a
+        return (int64_t)(std::upper_bound(cuts.begin(), cuts.end(), a) - cuts.begin());
+    };
+    int64_t c = 0;
+    while (c < cols) {
+        uintptr_t cl = lo + (uintptr_t)(c * hld * 8), ch = cl + (uintptr_t)(rows * 8);
+        if (segment(cl) != segment(ch - 1)) {
+            // this column straddles a boundary: 1D pieces
+            uintptr_t a = cl;
+            while (a < ch) {
+                auto it = std::upper_bound(cuts.begin(), cuts.end(), a);
+                uintptr_t b = (it == cuts.end() || *it > ch) ? ch : *it;
+                char *h = (char *)a;
+                char *d = (char *)(dev + c * dld) + (a - cl);
+                cudaError_t e = h2d ? cudaMemcpyAsync(d, h, b - a, kind, s) : cudaMemcpyAsync(h, d, b - a, kind, s);
+                if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync (tile piece)");
+                a = b;
+            }
+            ++c;
+            continue;
+        }
+        int64_t seg = segment(cl), c2 = c + 1;
+        while (c2 < cols) {
+            uintptr_t l2 = lo + (uintptr_t)(c2 * hld * 8), h2 = l2 + (uintptr_t)(rows * 8);
+            if (segment(l2) != seg || segment(h2 - 1) != seg) break;
+            ++c2;
+        }
+        int rc = cp2d(c, c2 - c);
+        if (rc) return rc;
+        c = c2;
+    }
+    return XK_OK;
+}
+
+static bool host_pinned(uintptr_t addr) {
+    cudaPointerAttributes a{};
+    bool ok = cudaPointerGetAttributes(&a, (void *)addr) == cudaSuccess && a.type == cudaMemoryTypeHost;
+    cudaGetLastError();
+    return ok;
+}
+
+// Page-lock a host view for the duration of the call (or of the async epoch).  Memory the
+// caller registered (xk_register, cudaHostRegister, cudaMallocHost, torch pin_memory) is
+// used as is; otherwise the page range is registered internally -- skipping a boundary
+// page that a neighbouring allocation already pinned -- and counted in the stats.  Internal
+// registrations are dropped at the next full synchronisation point, so a registration
+// never outlives the caller's buffer (the async contract keeps buffers alive until then).
+int Runtime::ensure_pinned(uint64_t base, int64_t rows, int64_t cols, int64_t ld) {
+    if (rows <= 0 || cols <= 0) return XK_OK;
+    uintptr_t lo = (uintptr_t)base, hi = lo + (uintptr_t)(((cols - 1) * ld + rows) * 8);
+    auto covered = [&](const std::map<uintptr_t, size_t> &m) {
+        auto it = m.upper_bound(lo);
+        if (it == m.begin()) return false;
+        --it;
+        return it->first <= lo && hi <= it->first + it->second;
+    };
+    if (covered(registered_) || covered(internal_reg_)) return XK_OK;
+    const uintptr_t page = 4096;
+    bool lo_p = host_pinned(lo), hi_p = host_pinned(hi - 1);
+    if (lo_p && hi_p && host_pinned(lo + (hi - lo) / 2)) return XK_OK;  // pinned elsewhere
+    uintptr_t plo = lo_p ? ((lo / page) + 1) * page : (lo / page) * page;
+    uintptr_t phi = hi_p ? ((hi - 1) / page) * page : ((hi + page - 1) / page) * page;
+    if (phi <= plo) return XK_OK;
+    cudaError_t e = cudaHostRegister((void *)plo, phi - plo, cudaHostRegisterPortable);
+    if (e == cudaErrorHostMemoryAlreadyRegistered) {
+        cudaGetLastError();
+        return XK_OK;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "cudaHostRegister (internal)");
+    internal_reg_[plo] = phi - plo;
+    stats.host_registrations++;
+    return XK_OK;
+}
+
+void Runtime::release_internal_pins() {
+    for (auto &kv : internal_reg_) cudaHostUnregister((void *)kv.first);
+    cudaGetLastError();
+    internal_reg_.clear();
+}
+
+int Runtime::register_host(void *p, size_t bytes, bool internal) {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    (void)internal;
+    if (!p || bytes == 0) return XK_OK;
+    cudaError_t e = cudaHostRegister(p, bytes, cudaHostRegisterPortable);
+    if (e == cudaErrorHostMemoryAlreadyRegistered) {
+        cudaGetLastError();
+        return XK_OK;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "cudaHostRegister");
+    registered_[(uintptr_t)p] = bytes;
+    return XK_OK;
+}
+
+int Runtime::unregister_host(void *p) {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    auto it = registered_.find((uintptr_t)p);
+    if (it == registered_.end()) return XK_OK;
+    int rc = sync_all();
+    if (rc) return rc;
+    registered_.erase(it);
+    XK_CK(cudaHostUnregister(p));
+    return XK_OK;
+}
+
+void Runtime::release_invalid() {
+    for (auto it = bufs_.begin(); it != bufs_.end();) {
+        int key = (int)(it->first / XK_MAX_GPUS), g = (int)(it->first % XK_MAX_GPUS);
+        if (!planner_->entry(key).gpu[g].present) {
+            free_buf(g, it->second.p, it->second.bytes);
+            it = bufs_.erase(it);
+        } else {
+            ++it;
+        }
+    }
+}
+
+int Runtime::sync_all() {
+    for (size_t g = 0; g < devs_.size(); ++g) {
+        Device &d = devs_[g];
+        XK_CK(cudaSetDevice(d.phys));
+        XK_CK(cudaStreamSynchronize(d.h2d));
+        XK_CK(cudaStreamSynchronize(d.p2p));
+        for (int k = 0; k < cfg_.kstreams; ++k) XK_CK(cudaStreamSynchronize(d.ks[k]));
+        XK_CK(cudaStreamSynchronize(d.d2h));
+    }
+    cur_dev_ = -1;
+    for (auto &t : ktimers_) {
+        float ms = 0;
+        if (cudaEventElapsedTime(&ms, t.first, t.second) == cudaSuccess) stats.kernel_ms_total += ms;
+        cudaEventDestroy(t.first);
+        cudaEventDestroy(t.second);
+    }
+    ktimers_.clear();
+    // every event of this epoch completed: recycle them
+    seq_ev_.clear();
+    pending_d2h_.clear();
+    for (auto &kv : bufs_) {
+        kv.second.writer = Ev();
+        kv.second.readers.clear();
+    }
+    for (size_t g = 0; g < devs_.size(); ++g) {
+        for (cudaEvent_t e : ev_used_[g]) ev_pool_[g].push_back(e);
+        ev_used_[g].clear();
+    }
+    release_internal_pins();
+    return XK_OK;
+}
+
+int Runtime::run(const xk_call_t &call, bool wait) {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    cur_dev_ = -1;
+    int rc;
+    // page-lock the operands the call touches (excluded from timings when the caller
+    // registered them first with xk_register)
+    if (call.routine == XK_ROUTINE_DGEMM) {
+        bool ta = call.transA == 'T' || call.transA == 'C', tb = call.transB == 'T' || call.transB == 'C';
+        if (call.alpha != 0.0 && call.k > 0) {
+            if ((rc = ensure_pinned(call.A, ta ? call.k : call.m, ta ? call.m : call.k, (int64_t)call.lda))) return rc;
+            if ((rc = ensure_pinned(call.B, tb ? call.n : call.k, tb ? call.k : call.n, (int64_t)call.ldb))) return rc;
+        }
+    }
+    if ((rc = ensure_pinned(call.C, call.m, call.n, (int64_t)call.ldc))) return rc;
+    std::vector<Rec> recs;
+    std::string err;
+    rc = planner_->plan(call, recs, err);
+    if (rc) {
+        set_error(err);
+        return rc;
+    }
+    size_t d2h0 = pending_d2h_.size();
+    for (const Rec &r : recs)
+        if ((rc = issue(r))) return rc;
+    if (call.routine == XK_ROUTINE_DGEMM && call.sync) {
+        // the planner already passed its full sync point and invalidated the operands
+        if ((rc = sync_all())) return rc;
+        release_invalid();
+        return XK_OK;
+    }
+    if (wait) {
+        for (size_t q = d2h0; q < pending_d2h_.size(); ++q) XK_CK(cudaEventSynchronize(pending_d2h_[q].e));
+    }
+    return XK_OK;
+}
+
+int Runtime::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    int rc = sync_all();
+    if (rc) return rc;
+    xk_call_t c{};
+    c.routine = XK_ROUTINE_SYNC;
+    std::vector<Rec> recs;
+    std::string err;
+    planner_->plan(c, recs, err);
+    planner_->invalidate(base, m, n, ld);
+    release_invalid();
+    return XK_OK;
+}
+
+int Runtime::finalize() {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    int rc = sync_all();
+    for (size_t g = 0; g < devs_.size(); ++g) {
+        Device &d = devs_[g];
+        cudaSetDevice(d.phys);
+        for (auto &pb : d.all_bufs) cudaFree(pb.first);
+        d.all_bufs.clear();
+        d.free_bufs.clear();
+        cudaStreamDestroy(d.h2d);
+        cudaStreamDestroy(d.d2h);
+        cudaStreamDestroy(d.p2p);
+        for (int k = 0; k < cfg_.kstreams; ++k) cudaStreamDestroy(d.ks[k]);
+        for (cudaEvent_t e : ev_pool_[g]) cudaEventDestroy(e);
+    }
+    bufs_.clear();
+    release_internal_pins();
+    for (auto &kv : registered_) cudaHostUnregister((void *)kv.first);
+    registered_.clear();
+    planner_.reset();
+    devs_.clear();
+    return rc;
+}
+
+}  // namespace xk

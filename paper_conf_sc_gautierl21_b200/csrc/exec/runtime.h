@@ -1,0 +1,105 @@
+// runtime.h -- the executor behind the C ABI: logical GPUs, per-GPU streams (one H2D, one
+// D2H, one P2P-in, k kernel streams -- "one stream per operation type", PAPER.md
+// P:316-321), the device tile cache (compact column-major tiles), events for
+// the plan's point-to-point dependencies, and the issue loop that turns plan
+// records into cudaMemcpy2DAsync / peer copies / tile-kernel launches.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "plan/plan.h"
+#include "xk.h"
+
+namespace xk {
+
+constexpr int kMaxKStreams = 8;
+
+struct Ev {
+    cudaEvent_t e = nullptr;
+    cudaStream_t s = nullptr;  // stream it was recorded on
+};
+
+// A device tile: compact column-major, ld = rows rounded up to 16 (128-byte columns).
+struct Buffer {
+    double *p = nullptr;
+    int64_t ld = 0;
+    size_t bytes = 0;
+    Ev writer;                  // last write (copy in or task)
+    std::vector<Ev> readers;    // reads since the last write (tasks, P2P out, D2H)
+};
+
+struct Device {
+    int phys = 0;
+    cudaStream_t h2d = nullptr, d2h = nullptr, p2p = nullptr;
+    cudaStream_t ks[kMaxKStreams] = {};
+    std::map<size_t, std::vector<double *>> free_bufs;  // caching allocator
+    std::vector<std::pair<double *, size_t>> all_bufs;
+    size_t bytes_in_use = 0;
+};
+
+class Runtime {
+public:
+    Runtime() = default;
+    ~Runtime();
+    int init(const xk_config_t &cfg);
+    int finalize();
+
+    // One planned call: plan, issue in plan order; `wait` = block until the D2H records
+    // of this call completed.  Sync routines pass call.sync = 1 and then release the
+    // device copies the planner invalidated.
+    int run(const xk_call_t &call, bool wait);
+    int sync_all();
+    int invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld);
+
+    int register_host(void *p, size_t bytes, bool internal);
+    int unregister_host(void *p);
+    int ensure_pinned(uint64_t base, int64_t rows, int64_t cols, int64_t ld);
+
+    xk_stats_t stats{};
+    bool kernel_timing = false;
+    Topology topo;
+    std::vector<int> perf_rank;
+    std::recursive_mutex mu;
+
+private:
+    int issue(const Rec &r);
+    Buffer *buf(int key, int g, bool create, int *rc);
+    void release_invalid();
+    cudaEvent_t new_event(int g);
+    int wait_on(cudaStream_t s, const Ev &ev);
+    int record(cudaStream_t s, int g, Ev *out);
+    int wait_dep(cudaStream_t s, int64_t seq);
+    int cuda_fail(cudaError_t e, const char *what);
+    double *alloc(int g, size_t bytes, int *rc);
+    void free_buf(int g, double *p, size_t bytes);
+    int probe_topology();
+    void release_internal_pins();
+    std::vector<uintptr_t> reg_cuts(uintptr_t lo, uintptr_t hi) const;
+    int copy_host(bool h2d, double *dev, int64_t dld, char *host, int64_t hld, int64_t rows,
+                  int64_t cols, cudaStream_t s);
+    int set_dev(int g);
+
+    xk_config_t cfg_{};
+    Flags flags_;
+    std::unique_ptr<Planner> planner_;
+    std::vector<Device> devs_;
+    std::unordered_map<int64_t, Buffer> bufs_;  // key * XK_MAX_GPUS + g
+    std::unordered_map<int64_t, Ev> seq_ev_;    // plan seq -> completion event (this epoch)
+    std::vector<std::vector<cudaEvent_t>> ev_pool_, ev_used_;  // per logical GPU
+    std::vector<Ev> pending_d2h_;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ktimers_;
+    std::map<uintptr_t, size_t> registered_;    // user-registered host ranges
+    std::map<uintptr_t, size_t> internal_reg_;  // registered by the library on first use
+    int cur_dev_ = -1;
+};
+
+Runtime *runtime();  // global instance (nullptr before xk_init)
+
+}  // namespace xk
