@@ -169,9 +169,11 @@ typedef struct xk_stats {
     int64_t flops[XK_MAX_GPUS];
     int64_t forwards_inflight;       /* P2P copies sourced from an in-flight copy (A2) */
     int64_t forwards_valid;          /* P2P copies sourced from a valid copy (A1) */
-    int64_t kernel_launches;
+    int64_t kernel_launches;         /* tile-kernel launches (one grouped launch per batch) */
     int64_t host_registrations;      /* unregistered host ranges registered internally */
-    double kernel_ms_total;          /* summed dgemm tile-kernel time (when timing on) */
+    double kernel_ms_total;          /* summed tile-kernel launch time (when timing on) */
+    int64_t kernel_timed_launches;   /* launches included in kernel_ms_total */
+    int64_t kernel_timed_flops;      /* algorithmic flops of those launches (2*m*n*k per task) */
 } xk_stats_t;
 int xk_get_stats(xk_stats_t *out);
 int xk_reset_stats(void);

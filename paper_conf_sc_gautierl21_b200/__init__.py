@@ -166,7 +166,7 @@ def get_stats():
     for f in ("h2d_bytes", "d2h_bytes", "p2p_in_bytes", "p2p_out_bytes", "tasks", "flops"):
         out[f] = list(getattr(st, f))[:G]
     for f in ("forwards_inflight", "forwards_valid", "kernel_launches", "host_registrations",
-              "kernel_ms_total"):
+              "kernel_ms_total", "kernel_timed_launches", "kernel_timed_flops"):
         out[f] = getattr(st, f)
     return out
 

@@ -44,7 +44,8 @@ class Stats(ctypes.Structure):
                 ("p2p_in_bytes", i64 * MAX_GPUS), ("p2p_out_bytes", i64 * MAX_GPUS),
                 ("tasks", i64 * MAX_GPUS), ("flops", i64 * MAX_GPUS),
                 ("forwards_inflight", i64), ("forwards_valid", i64), ("kernel_launches", i64),
-                ("host_registrations", i64), ("kernel_ms_total", c_double)]
+                ("host_registrations", i64), ("kernel_ms_total", c_double),
+                ("kernel_timed_launches", i64), ("kernel_timed_flops", i64)]
 
 
 class Topo(ctypes.Structure):

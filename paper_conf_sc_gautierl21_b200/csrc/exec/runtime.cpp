@@ -90,6 +90,13 @@ int Runtime::init(const xk_config_t &cfg) {
     cur_dev_ = -1;
     ev_pool_.assign(G, {});
     ev_used_.assign(G, {});
+    batch_.assign(G, PendingBatch());
+    batch_count_.assign(G, 0);
+    {
+        const char *eb = std::getenv("XK_BATCH");
+        int mb = (eb && *eb) ? std::atoi(eb) : kMaxBatch;
+        max_batch_ = std::max(1, std::min(kMaxBatch, mb));
+    }
     // flags
     flags_.topo = cfg.topo;
     flags_.optimistic = cfg.optimistic;
@@ -330,6 +337,7 @@ int Runtime::issue(const Rec &R) {
     const Matrix &M = planner_->matrix(e.mat);
     const int64_t T = flags_.T;
     int rc = XK_OK;
+    if (r.kind != XK_REC_TASK && (rc = flush_for(R))) return rc;
     switch (r.kind) {
     case XK_REC_H2D: {
         const int g = r.dst;
@@ -384,50 +392,42 @@ int Runtime::issue(const Rec &R) {
         if ((rc = set_dev(g))) return rc;
         Buffer *O = buf(R.key, g, true, &rc);
         if (!O) return rc;
-        Buffer *A = nullptr, *B = nullptr;
-        if (R.keyA >= 0) {
-            if (!(A = buf(R.keyA, g, false, &rc))) return rc;
-            if (!(B = buf(R.keyB, g, false, &rc))) return rc;
-            O = buf(R.key, g, false, &rc);
+        const int64_t idO = (int64_t)R.key * XK_MAX_GPUS + g;
+        if (R.keyA < 0) {  // scale-only task (alpha == 0 or k == 0): not batched
+            if ((rc = flush_batch(g))) return rc;
+            cudaStream_t s = devs_[g].ks[0];
+            for (int q = 0; q < 4; ++q)
+                if ((rc = wait_dep(s, r.dep[q]))) return rc;
+            for (auto &rd : O->readers)
+                if ((rc = wait_on(s, rd))) return rc;
+            if ((rc = wait_on(s, O->writer))) return rc;
+            cudaError_t ke = launch_scale_tile(R.m, R.n, R.beta, O->p, O->ld, s);
+            if (ke != cudaSuccess) return cuda_fail(ke, "scale kernel launch");
+            Ev ev;
+            if ((rc = record(s, g, &ev))) return rc;
+            seq_ev_[r.seq] = ev;
+            O->writer = ev;
+            O->readers.clear();
+            stats.tasks[g]++;
+            stats.flops[g] += r.work;
+            stats.kernel_launches++;
+            return XK_OK;
         }
-        const Device &d = devs_[g];
-        uint64_t h = (uint64_t)(e.bi * 7919 + e.bj * 104729);
-        cudaStream_t s = d.ks[h % (uint64_t)cfg_.kstreams];
-        for (int q = 0; q < 4; ++q)
-            if ((rc = wait_dep(s, r.dep[q]))) return rc;
-        for (auto &rd : O->readers)
-            if ((rc = wait_on(s, rd))) return rc;
-        if ((rc = wait_on(s, O->writer))) return rc;
-        cudaEvent_t t0 = nullptr, t1 = nullptr;
-        if (kernel_timing) {
-            XK_CK(cudaEventCreate(&t0));
-            XK_CK(cudaEventCreate(&t1));
-            XK_CK(cudaEventRecord(t0, s));
-        }
-        cudaError_t ke;
-        if (A) {
-            ke = launch_dgemm_tile(R.ta == 'T', R.tb == 'T', R.m, R.n, R.k, R.alpha, A->p, A->ld,
-                                   B->p, B->ld, R.beta, O->p, O->ld, s);
-        } else {
-            ke = launch_scale_tile(R.m, R.n, R.beta, O->p, O->ld, s);
-        }
-        if (ke != cudaSuccess) return cuda_fail(ke, "tile kernel launch");
-        if (kernel_timing) {
-            XK_CK(cudaEventRecord(t1, s));
-            ktimers_.push_back({t0, t1});
-        }
-        Ev ev;
-        if ((rc = record(s, g, &ev))) return rc;
-        seq_ev_[r.seq] = ev;
-        O->writer = ev;
-        O->readers.clear();
-        if (A) {
-            add_reader(*A, ev);
-            add_reader(*B, ev);
-        }
-        stats.tasks[g]++;
-        stats.flops[g] += r.work;
-        stats.kernel_launches++;
+        if (!buf(R.keyA, g, false, &rc) || !buf(R.keyB, g, false, &rc)) return rc;
+        const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g, idB = (int64_t)R.keyB * XK_MAX_GPUS + g;
+        PendingBatch &bt = batch_[g];
+        bool conflict = (int)bt.recs.size() >= max_batch_ ||
+                        (!bt.recs.empty() && (bt.ta != R.ta || bt.tb != R.tb)) ||
+                        bt.touches(idO, true) || bt.touches(idA, false) || bt.touches(idB, false);
+        for (int q = 0; q < 4 && !conflict; ++q)
+            if (r.dep[q] >= 0 && bt.contains_seq(r.dep[q])) conflict = true;
+        if (conflict && (rc = flush_batch(g))) return rc;
+        bt.recs.push_back(&R);
+        bt.out_ids.push_back(idO);
+        bt.in_ids.push_back(idA);
+        bt.in_ids.push_back(idB);
+        bt.ta = R.ta;
+        bt.tb = R.tb;
         return XK_OK;
     }
     case XK_REC_D2H: {
@@ -454,6 +454,84 @@ int Runtime::issue(const Rec &R) {
         set_error("internal: unknown record kind");
         return XK_ERR_INTERNAL;
     }
+}
+
+// Launch the pending tile tasks of GPU g as one grouped kernel on the next kernel stream.
+int Runtime::flush_batch(int g) {
+    PendingBatch &bt = batch_[g];
+    if (bt.recs.empty()) return XK_OK;
+    int rc;
+    if ((rc = set_dev(g))) return rc;
+    const Device &d = devs_[g];
+    cudaStream_t s = d.ks[batch_count_[g]++ % cfg_.kstreams];
+    TileBatch tb;
+    tb.n = (int)bt.recs.size();
+    int64_t flops = 0;
+    for (int q = 0; q < tb.n; ++q) {
+        const Rec &R = *bt.recs[q];
+        for (int j = 0; j < 4; ++j)
+            if ((rc = wait_dep(s, R.r.dep[j]))) return rc;
+        Buffer *O = buf(R.key, g, false, &rc);
+        Buffer *A = buf(R.keyA, g, false, &rc);
+        Buffer *B = buf(R.keyB, g, false, &rc);
+        if (!O || !A || !B) return rc;
+        for (auto &rd : O->readers)
+            if ((rc = wait_on(s, rd))) return rc;
+        if ((rc = wait_on(s, O->writer))) return rc;
+        tb.t[q] = TileTask{A->p, B->p, O->p, A->ld, B->ld, O->ld, R.m, R.n, R.k, R.alpha, R.beta};
+        flops += R.r.work;
+    }
+    cudaEvent_t t0 = nullptr, t1 = nullptr;
+    if (kernel_timing) {
+        XK_CK(cudaEventCreate(&t0));
+        XK_CK(cudaEventCreate(&t1));
+        XK_CK(cudaEventRecord(t0, s));
+    }
+    cudaError_t ke = launch_dgemm_batch(bt.ta == 'T', bt.tb == 'T', tb, s);
+    if (ke != cudaSuccess) return cuda_fail(ke, "tile kernel launch");
+    if (kernel_timing) {
+        XK_CK(cudaEventRecord(t1, s));
+        ktimers_.push_back({t0, t1});
+        ktimer_flops_.push_back(flops);
+    }
+    Ev ev;
+    if ((rc = record(s, g, &ev))) return rc;
+    for (int q = 0; q < tb.n; ++q) {
+        const Rec &R = *bt.recs[q];
+        seq_ev_[R.r.seq] = ev;
+        Buffer *O = buf(R.key, g, false, &rc);
+        O->writer = ev;
+        O->readers.clear();
+        add_reader(*buf(R.keyA, g, false, &rc), ev);
+        add_reader(*buf(R.keyB, g, false, &rc), ev);
+        stats.tasks[g]++;
+        stats.flops[g] += R.r.work;
+    }
+    stats.kernel_launches++;
+    bt.recs.clear();
+    bt.out_ids.clear();
+    bt.in_ids.clear();
+    return XK_OK;
+}
+
+// Before a copy record is issued: launch any pending batch it depends on or whose
+// buffers it overwrites.
+int Runtime::flush_for(const Rec &R) {
+    const xk_plan_rec_t &r = R.r;
+    for (size_t g = 0; g < batch_.size(); ++g) {
+        PendingBatch &bt = batch_[g];
+        if (bt.recs.empty()) continue;
+        bool need = r.dep[0] >= 0 && bt.contains_seq(r.dep[0]);
+        if (!need && r.kind != XK_REC_D2H && r.dst == (int)g)
+            need = bt.touches((int64_t)R.key * XK_MAX_GPUS + g, true);
+        if (!need && (r.kind == XK_REC_P2P || r.kind == XK_REC_D2H) && r.src == (int)g)
+            need = bt.touches((int64_t)R.key * XK_MAX_GPUS + g, false);
+        if (need) {
+            int rc = flush_batch((int)g);
+            if (rc) return rc;
+        }
+    }
+    return XK_OK;
 }
 
 // Boundaries of host registrations strictly inside [lo, hi): a pinned copy must not
@@ -619,13 +697,18 @@ int Runtime::sync_all() {
         XK_CK(cudaStreamSynchronize(d.d2h));
     }
     cur_dev_ = -1;
-    for (auto &t : ktimers_) {
+    for (size_t q = 0; q < ktimers_.size(); ++q) {
         float ms = 0;
-        if (cudaEventElapsedTime(&ms, t.first, t.second) == cudaSuccess) stats.kernel_ms_total += ms;
-        cudaEventDestroy(t.first);
-        cudaEventDestroy(t.second);
+        if (cudaEventElapsedTime(&ms, ktimers_[q].first, ktimers_[q].second) == cudaSuccess) {
+            stats.kernel_ms_total += ms;
+            stats.kernel_timed_flops += ktimer_flops_[q];
+            stats.kernel_timed_launches++;
+        }
+        cudaEventDestroy(ktimers_[q].first);
+        cudaEventDestroy(ktimers_[q].second);
     }
     ktimers_.clear();
+    ktimer_flops_.clear();
     // every event of this epoch completed: recycle them
     seq_ev_.clear();
     pending_d2h_.clear();
@@ -665,6 +748,8 @@ int Runtime::run(const xk_call_t &call, bool wait) {
     size_t d2h0 = pending_d2h_.size();
     for (const Rec &r : recs)
         if ((rc = issue(r))) return rc;
+    for (size_t g = 0; g < batch_.size(); ++g)
+        if ((rc = flush_batch((int)g))) return rc;
     if (call.routine == XK_ROUTINE_DGEMM && call.sync) {
         // the planner already passed its full sync point and invalidated the operands
         if ((rc = sync_all())) return rc;

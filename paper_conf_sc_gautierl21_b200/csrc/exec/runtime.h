@@ -14,6 +14,7 @@
 #include <unordered_map>
 #include <vector>
 
+#include "kernels/kernels.h"
 #include "plan/plan.h"
 #include "xk.h"
 
@@ -33,6 +34,26 @@ struct Buffer {
     size_t bytes = 0;
     Ev writer;                  // last write (copy in or task)
     std::vector<Ev> readers;    // reads since the last write (tasks, P2P out, D2H)
+};
+
+// Tile tasks of one GPU waiting to be launched together (grouped GEMM launch).
+struct PendingBatch {
+    std::vector<const Rec *> recs;
+    std::vector<int64_t> out_ids, in_ids;  // buffer ids written / read
+    char ta = 'N', tb = 'N';
+    bool contains_seq(int64_t seq) const {
+        for (const Rec *r : recs)
+            if (r->r.seq == seq) return true;
+        return false;
+    }
+    bool touches(int64_t id, bool write) const {
+        for (int64_t o : out_ids)
+            if (o == id) return true;
+        if (write)
+            for (int64_t i : in_ids)
+                if (i == id) return true;
+        return false;
+    }
 };
 
 struct Device {
@@ -70,6 +91,8 @@ public:
 
 private:
     int issue(const Rec &r);
+    int flush_batch(int g);
+    int flush_for(const Rec &r);
     Buffer *buf(int key, int g, bool create, int *rc);
     void release_invalid();
     cudaEvent_t new_event(int g);
@@ -95,9 +118,13 @@ private:
     std::vector<std::vector<cudaEvent_t>> ev_pool_, ev_used_;  // per logical GPU
     std::vector<Ev> pending_d2h_;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ktimers_;
+    std::vector<int64_t> ktimer_flops_;
     std::map<uintptr_t, size_t> registered_;    // user-registered host ranges
     std::map<uintptr_t, size_t> internal_reg_;  // registered by the library on first use
     int cur_dev_ = -1;
+    std::vector<PendingBatch> batch_;
+    std::vector<int64_t> batch_count_;
+    int max_batch_ = kMaxBatch;
 };
 
 Runtime *runtime();  // global instance (nullptr before xk_init)

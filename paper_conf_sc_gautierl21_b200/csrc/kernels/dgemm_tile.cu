@@ -13,32 +13,33 @@
 // on DMMA.  Operands are staged through a multi-stage cp.async (LDGSTS) shared-memory
 // ring with zero-fill predication for ragged edges; fragments are read with
 // conflict-free padded strides; alpha/beta are fused into the register epilogue.
+//
+// One launch runs a BATCH of up to kMaxBatch independent tile tasks (grouped GEMM): the
+// executor groups ready tasks of one GPU so a launch is many waves long -- no per-task
+// wave-quantization tail (a single T=2048 task is only 1.7 waves on 148 SMs) and one
+// launch per batch instead of per task.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "kernels/kernels.h"
 
 namespace xk {
 namespace {
 
-constexpr int BK = 16;          // k per pipeline stage
-constexpr int PAD_MN = 4;       // [k][mn] layout: stride BM+4 doubles (2*stride = 8 mod 32 words)
-constexpr int STRIDE_K = 20;    // [mn][k] layout: stride 16+4 doubles
+constexpr int PAD_MN = 4;  // [k][mn] layout: stride BMN+4 doubles (2*stride = 8 mod 32 words)
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
 template <int VEC>
-__device__ __forceinline__ void cp_async(double *dst, const double *src, int valid) {
+__device__ __forceinline__ void cp_async(uint32_t dst, const double *src, int valid) {
     // copy `valid` of VEC doubles, zero-fill the rest (src-size operand)
-    uint32_t d = smem_u32(dst);
     if constexpr (VEC == 2) {
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src),
-                     "r"(valid * 8));
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst), "l"(src), "r"(valid * 8));
     } else {
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src),
-                     "r"(valid * 8));
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(dst), "l"(src), "r"(valid * 8));
     }
 }
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::); }
@@ -51,55 +52,71 @@ __device__ __forceinline__ void dmma(double (&c)[2], double a, double b) {
                  : "d"(a), "d"(b));
 }
 
-// Shared-memory footprint of one operand slab (BMN x BK) in doubles.
-template <int BMN, bool MN_CONTIG>
+// Shared-memory slab of op(X), BMN x BK doubles.  MN_CONTIG: stored [k][mn] (mn
+// contiguous, stride BMN+4); else [mn][k] (k contiguous, stride BK+4).  Both strides give
+// conflict-free 8-byte fragment reads for the m8n8k4 A/B fragments.
+template <int BMN, bool MN_CONTIG, int BK>
 struct Slab {
-    static constexpr int kStride = MN_CONTIG ? (BMN + PAD_MN) : STRIDE_K;
-    static constexpr int kDoubles = MN_CONTIG ? BK * (BMN + PAD_MN) : BMN * STRIDE_K;
+    static constexpr int kStride = MN_CONTIG ? (BMN + PAD_MN) : (BK + 4);
+    static constexpr int kDoubles = MN_CONTIG ? BK * (BMN + PAD_MN) : BMN * (BK + 4);
     __device__ __forceinline__ static int idx(int mn, int k) {
         return MN_CONTIG ? k * kStride + mn : mn * kStride + k;
     }
 };
 
-// Load a BMN x BK slab of op(X) into shared memory.  Global element (mn, k) of op(X) is
-// X[mn + k*ld] when MN_CONTIG (mn contiguous) else X[k + mn*ld].
-template <int BMN, bool MN_CONTIG, int VEC, int NTHREADS>
-__device__ __forceinline__ void load_slab(double *s, const double *X, int64_t ld, int64_t mn0,
-                                          int64_t k0, int64_t MN, int64_t K, int tid) {
-    using S = Slab<BMN, MN_CONTIG>;
-    constexpr int kChunks = BMN * BK / VEC;
-    static_assert(kChunks % NTHREADS == 0, "chunking");
-#pragma unroll
-    for (int q = 0; q < kChunks / NTHREADS; ++q) {
-        int c = tid + q * NTHREADS;
-        int mn, k;
-        int64_t gm, gk;
-        int valid;
+// Loader of one operand slab: a thread's chunks keep the same (mn, k) slab coordinates
+// every stage; interior blocks skip the ragged-edge predication entirely.
+template <int BMN, bool MN_CONTIG, int BK, int VEC, int NTHREADS>
+struct Loader {
+    using S = Slab<BMN, MN_CONTIG, BK>;
+    static constexpr int kChunks = BMN * BK / VEC / NTHREADS;  // chunks per thread
+    static_assert(BMN * BK / VEC % NTHREADS == 0, "chunking");
+    const double *base;
+    int64_t ld, MN, K, mn0;
+
+    __device__ __forceinline__ static void coords(int c, int &mn, int &k) {
         if (MN_CONTIG) {
             k = c / (BMN / VEC);
             mn = (c % (BMN / VEC)) * VEC;
-            gm = mn0 + mn;
-            gk = k0 + k;
-            int64_t rem = MN - gm;
-            valid = (gk < K && rem > 0) ? (int)(rem < VEC ? rem : VEC) : 0;
         } else {
             mn = c / (BK / VEC);
             k = (c % (BK / VEC)) * VEC;
-            gm = mn0 + mn;
-            gk = k0 + k;
-            int64_t rem = K - gk;
-            valid = (gm < MN && rem > 0) ? (int)(rem < VEC ? rem : VEC) : 0;
         }
-        const double *src = valid ? (MN_CONTIG ? X + gm + gk * ld : X + gk + gm * ld) : X;
-        cp_async<VEC>(s + S::idx(mn, k), src, valid);
     }
-}
+    __device__ __forceinline__ void init(const double *X, int64_t ld_, int64_t mn0_, int64_t MN_,
+                                         int64_t K_) {
+        base = X;
+        ld = ld_;
+        mn0 = mn0_;
+        MN = MN_;
+        K = K_;
+    }
+    // issue the copies of the k-block starting at k0 into the slab at shared address s
+    __device__ __forceinline__ void load(uint32_t s, int64_t k0, int tid, bool interior) const {
+#pragma unroll
+        for (int q = 0; q < kChunks; ++q) {
+            int mn, k;
+            coords(tid + q * NTHREADS, mn, k);
+            const int64_t gm = mn0 + mn, gk = k0 + k;
+            int valid;
+            if (interior) {
+                valid = VEC;
+            } else if (MN_CONTIG) {
+                const int64_t rem = MN - gm;
+                valid = (gk < K && rem > 0) ? (int)(rem < VEC ? rem : VEC) : 0;
+            } else {
+                const int64_t rem = K - gk;
+                valid = (gm < MN && rem > 0) ? (int)(rem < VEC ? rem : VEC) : 0;
+            }
+            const double *src = valid ? (MN_CONTIG ? base + gm + gk * ld : base + gk + gm * ld) : base;
+            cp_async<VEC>(s + 8u * (uint32_t)S::idx(mn, k), src, valid);
+        }
+    }
+};
 
-template <int BM, int BN, int WM, int WN, int STAGES, bool TA, bool TB, int VEC>
-__global__ void __launch_bounds__((BM / WM) * (BN / WN) * 32, 1)
-dgemm_tile_kernel(int64_t M, int64_t N, int64_t K, double alpha, const double *__restrict__ A,
-                  int64_t lda, const double *__restrict__ B, int64_t ldb, double beta,
-                  double *__restrict__ C, int64_t ldc) {
+template <int BM, int BN, int WM, int WN, int BK, int STAGES, int MINB, bool TA, bool TB, int VEC>
+__global__ void __launch_bounds__((BM / WM) * (BN / WN) * 32, MINB)
+dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
     constexpr int NWM = BM / WM, NWN = BN / WN;
     constexpr int NTHREADS = NWM * NWN * 32;
     constexpr int MF = WM / 8, NF = WN / 8;
@@ -107,18 +124,34 @@ dgemm_tile_kernel(int64_t M, int64_t N, int64_t K, double alpha, const double *_
     // B: op(B) is K x N; 'N' -> k contiguous, 'T' -> n contiguous.
     constexpr bool A_MN = !TA;
     constexpr bool B_MN = TB;
-    using SA = Slab<BM, A_MN>;
-    using SB = Slab<BN, B_MN>;
+    using SA = Slab<BM, A_MN, BK>;
+    using SB = Slab<BN, B_MN, BK>;
+
+    // which task of the batch, which CTA tile of it
+    int q = 0;
+    const int bid = blockIdx.x;
+#pragma unroll 1
+    while (q + 1 < batch.n && bid >= batch.cta_start[q + 1]) ++q;
+    const TileTask &t = batch.t[q];
+    const int local = bid - batch.cta_start[q];
+    const int tiles_m = (int)((t.M + BM - 1) / BM);
+    const int64_t m0 = (int64_t)(local % tiles_m) * BM, n0 = (int64_t)(local / tiles_m) * BN;
+    const int64_t M = t.M, N = t.N, K = t.K;
 
     extern __shared__ __align__(128) double smem[];
-    double *sA = smem;
-    double *sB = smem + STAGES * SA::kDoubles;
+    const uint32_t sA0 = smem_u32(smem);
+    const uint32_t sB0 = sA0 + 8u * STAGES * SA::kDoubles;
 
     const int tid = threadIdx.x;
     const int lane = tid & 31, warp = tid >> 5;
     const int wm = (warp % NWM) * WM, wn = (warp / NWM) * WN;
-    const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;
     const int KB = (int)((K + BK - 1) / BK);
+    const bool mn_interior = (m0 + BM <= M) && (n0 + BN <= N);
+
+    Loader<BM, A_MN, BK, VEC, NTHREADS> la;
+    Loader<BN, B_MN, BK, VEC, NTHREADS> lb;
+    la.init(t.A, t.lda, m0, M, K);
+    lb.init(t.B, t.ldb, n0, N, K);
 
     double acc[MF][NF][2];
 #pragma unroll
@@ -129,27 +162,34 @@ dgemm_tile_kernel(int64_t M, int64_t N, int64_t K, double alpha, const double *_
 #pragma unroll
     for (int s = 0; s < STAGES - 1; ++s) {
         if (s < KB) {
-            load_slab<BM, A_MN, VEC, NTHREADS>(sA + s * SA::kDoubles, A, lda, m0, (int64_t)s * BK, M, K, tid);
-            load_slab<BN, B_MN, VEC, NTHREADS>(sB + s * SB::kDoubles, B, ldb, n0, (int64_t)s * BK, N, K, tid);
+            const int64_t k0 = (int64_t)s * BK;
+            const bool in = mn_interior && (k0 + BK <= K);
+            la.load(sA0 + 8u * s * SA::kDoubles, k0, tid, in);
+            lb.load(sB0 + 8u * s * SB::kDoubles, k0, tid, in);
         }
         cp_commit();
     }
 
     const int fr = lane >> 2, fc = lane & 3;
+    const double *sAd = smem;
+    const double *sBd = smem + STAGES * SA::kDoubles;
+#pragma unroll 1
     for (int kb = 0; kb < KB; ++kb) {
         cp_wait<STAGES - 2>();
         __syncthreads();
         {
-            int nk = kb + STAGES - 1;
+            const int nk = kb + STAGES - 1;
             if (nk < KB) {
-                int st = nk % STAGES;
-                load_slab<BM, A_MN, VEC, NTHREADS>(sA + st * SA::kDoubles, A, lda, m0, (int64_t)nk * BK, M, K, tid);
-                load_slab<BN, B_MN, VEC, NTHREADS>(sB + st * SB::kDoubles, B, ldb, n0, (int64_t)nk * BK, N, K, tid);
+                const int st = nk % STAGES;
+                const int64_t k0 = (int64_t)nk * BK;
+                const bool in = mn_interior && (k0 + BK <= K);
+                la.load(sA0 + 8u * st * SA::kDoubles, k0, tid, in);
+                lb.load(sB0 + 8u * st * SB::kDoubles, k0, tid, in);
             }
             cp_commit();
         }
-        const double *a = sA + (kb % STAGES) * SA::kDoubles;
-        const double *b = sB + (kb % STAGES) * SB::kDoubles;
+        const double *a = sAd + (kb % STAGES) * SA::kDoubles;
+        const double *b = sBd + (kb % STAGES) * SB::kDoubles;
 #pragma unroll
         for (int ks = 0; ks < BK; ks += 4) {
             double fa[MF], fb[NF];
@@ -166,15 +206,18 @@ dgemm_tile_kernel(int64_t M, int64_t N, int64_t K, double alpha, const double *_
     cp_wait<0>();
 
     // epilogue: D = alpha*acc + beta*C (C not read when beta == 0)
+    const double alpha = t.alpha, beta = t.beta;
+    double *C = t.C;
+    const int64_t ldc = t.ldc;
 #pragma unroll
     for (int i = 0; i < MF; ++i) {
-        int64_t r = m0 + wm + i * 8 + fr;
+        const int64_t r = m0 + wm + i * 8 + fr;
         if (r >= M) continue;
 #pragma unroll
         for (int j = 0; j < NF; ++j) {
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
-                int64_t c = n0 + wn + j * 8 + fc * 2 + h;
+                const int64_t c = n0 + wn + j * 8 + fc * 2 + h;
                 if (c >= N) continue;
                 double *p = C + r + c * ldc;
                 double v = alpha * acc[i][j][h];
@@ -185,14 +228,12 @@ dgemm_tile_kernel(int64_t M, int64_t N, int64_t K, double alpha, const double *_
     }
 }
 
-template <int BM, int BN, int WM, int WN, int STAGES, bool TA, bool TB, int VEC>
-cudaError_t launch_cfg(int64_t M, int64_t N, int64_t K, double alpha, const double *A,
-                       int64_t lda, const double *B, int64_t ldb, double beta, double *C,
-                       int64_t ldc, cudaStream_t st) {
-    using SA = Slab<BM, !TA>;
-    using SB = Slab<BN, TB>;
+template <int BM, int BN, int WM, int WN, int BK, int STAGES, int MINB, bool TA, bool TB, int VEC>
+cudaError_t launch_cfg(TileBatch &b, cudaStream_t st) {
+    using SA = Slab<BM, !TA, BK>;
+    using SB = Slab<BN, TB, BK>;
     constexpr size_t smem = (size_t)STAGES * (SA::kDoubles + SB::kDoubles) * sizeof(double);
-    auto kern = dgemm_tile_kernel<BM, BN, WM, WN, STAGES, TA, TB, VEC>;
+    auto kern = dgemm_tile_kernel<BM, BN, WM, WN, BK, STAGES, MINB, TA, TB, VEC>;
     static unsigned attr_set = 0;  // per instantiation, one bit per device (idempotent)
     int dev = 0;
     cudaGetDevice(&dev);
@@ -201,18 +242,43 @@ cudaError_t launch_cfg(int64_t M, int64_t N, int64_t K, double alpha, const doub
         if (e != cudaSuccess) return e;
         attr_set |= 1u << dev;
     }
-    dim3 grid((unsigned)((M + BM - 1) / BM), (unsigned)((N + BN - 1) / BN));
-    dim3 block((BM / WM) * (BN / WN) * 32);
-    kern<<<grid, block, smem, st>>>(M, N, K, alpha, A, lda, B, ldb, beta, C, ldc);
+    int total = 0;
+    for (int q = 0; q < b.n; ++q) {
+        b.cta_start[q] = total;
+        total += (int)(((b.t[q].M + BM - 1) / BM) * ((b.t[q].N + BN - 1) / BN));
+    }
+    b.cta_start[b.n] = total;
+    if (total == 0) return cudaSuccess;
+    kern<<<total, (BM / WM) * (BN / WN) * 32, smem, st>>>(b);
     return cudaGetLastError();
 }
 
+// Kernel configurations (tuning sweep via XK_KCFG; the default is the measured best).
+//   0: 128x128 CTA, 8 warps of 64x32, BK 16, 4 stages, 1 CTA/SM
+//   1: 128x64  CTA, 4 warps of 64x32, BK 16, 4 stages, 2 CTAs/SM (independent barriers)
+//   2: 128x128 CTA, 8 warps of 64x32, BK 32, 3 stages
+//   4: 128x64  CTA, 4 warps of 64x32, BK 16, 3 stages, 2 CTAs/SM  (default)
+int g_kcfg = -1;
+int kcfg() {
+    if (g_kcfg < 0) {
+        const char *e = getenv("XK_KCFG");
+        g_kcfg = (e && *e) ? atoi(e) : 4;
+    }
+    return g_kcfg;
+}
+
 template <bool TA, bool TB, int VEC>
-cudaError_t launch_t(int64_t M, int64_t N, int64_t K, double alpha, const double *A, int64_t lda,
-                     const double *B, int64_t ldb, double beta, double *C, int64_t ldc,
-                     cudaStream_t st) {
-    return launch_cfg<128, 128, 64, 32, 4, TA, TB, VEC>(M, N, K, alpha, A, lda, B, ldb, beta, C,
-                                                        ldc, st);
+cudaError_t launch_t(TileBatch &b, cudaStream_t st) {
+    switch (kcfg()) {
+    case 0:
+        return launch_cfg<128, 128, 64, 32, 16, 4, 1, TA, TB, VEC>(b, st);
+    case 1:
+        return launch_cfg<128, 64, 64, 32, 16, 4, 2, TA, TB, VEC>(b, st);
+    case 2:
+        return launch_cfg<128, 128, 64, 32, 32, 3, 1, TA, TB, VEC>(b, st);
+    default:
+        return launch_cfg<128, 64, 64, 32, 16, 3, 2, TA, TB, VEC>(b, st);
+    }
 }
 
 __global__ void scale_tile_kernel(int64_t M, int64_t N, double beta, double *C, int64_t ldc) {
@@ -227,24 +293,35 @@ __global__ void scale_tile_kernel(int64_t M, int64_t N, double beta, double *C, 
 
 }  // namespace
 
-cudaError_t launch_dgemm_tile(bool ta, bool tb, int64_t M, int64_t N, int64_t K, double alpha,
-                              const double *A, int64_t lda, const double *B, int64_t ldb,
-                              double beta, double *C, int64_t ldc, cudaStream_t st) {
-    if (M <= 0 || N <= 0) return cudaSuccess;
-    if (alpha == 0.0 || K <= 0) return launch_scale_tile(M, N, beta, C, ldc, st);
-    // 16-byte cp.async needs 16-byte aligned columns of both operands
-    bool v2 = ((lda | ldb) % 2 == 0) && (((uintptr_t)A | (uintptr_t)B) % 16 == 0);
-#define XK_DISPATCH(VEC)                                                                       \
-    if (!ta && !tb) return launch_t<false, false, VEC>(M, N, K, alpha, A, lda, B, ldb, beta, C, ldc, st); \
-    if (!ta && tb) return launch_t<false, true, VEC>(M, N, K, alpha, A, lda, B, ldb, beta, C, ldc, st);   \
-    if (ta && !tb) return launch_t<true, false, VEC>(M, N, K, alpha, A, lda, B, ldb, beta, C, ldc, st);   \
-    return launch_t<true, true, VEC>(M, N, K, alpha, A, lda, B, ldb, beta, C, ldc, st);
+cudaError_t launch_dgemm_batch(bool ta, bool tb, TileBatch &b, cudaStream_t st) {
+    if (b.n <= 0) return cudaSuccess;
+    // 16-byte cp.async needs 16-byte aligned columns of both operands in every task
+    bool v2 = true;
+    for (int q = 0; q < b.n; ++q)
+        v2 = v2 && ((b.t[q].lda | b.t[q].ldb) % 2 == 0) &&
+             ((((uintptr_t)b.t[q].A) | ((uintptr_t)b.t[q].B)) % 16 == 0);
+#define XK_DISPATCH(VEC)                                               \
+    if (!ta && !tb) return launch_t<false, false, VEC>(b, st);          \
+    if (!ta && tb) return launch_t<false, true, VEC>(b, st);            \
+    if (ta && !tb) return launch_t<true, false, VEC>(b, st);            \
+    return launch_t<true, true, VEC>(b, st);
     if (v2) {
         XK_DISPATCH(2)
     } else {
         XK_DISPATCH(1)
     }
 #undef XK_DISPATCH
+}
+
+cudaError_t launch_dgemm_tile(bool ta, bool tb, int64_t M, int64_t N, int64_t K, double alpha,
+                              const double *A, int64_t lda, const double *B, int64_t ldb,
+                              double beta, double *C, int64_t ldc, cudaStream_t st) {
+    if (M <= 0 || N <= 0) return cudaSuccess;
+    if (alpha == 0.0 || K <= 0) return launch_scale_tile(M, N, beta, C, ldc, st);
+    TileBatch b;
+    b.n = 1;
+    b.t[0] = TileTask{A, B, C, lda, ldb, ldc, M, N, K, alpha, beta};
+    return launch_dgemm_batch(ta, tb, b, st);
 }
 
 cudaError_t launch_scale_tile(int64_t M, int64_t N, double beta, double *C, int64_t ldc,

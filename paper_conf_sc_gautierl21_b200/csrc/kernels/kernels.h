@@ -4,7 +4,29 @@
 #include <stdint.h>
 
 namespace xk {
-// D = alpha*op(A)*op(B) + beta*C on column-major device tiles (dgemm_tile.cu).
+
+// One tile task D = alpha*op(A)*op(B) + beta*C on column-major device tiles.
+struct TileTask {
+    const double *A;
+    const double *B;
+    double *C;
+    int64_t lda, ldb, ldc;
+    int64_t M, N, K;
+    double alpha, beta;
+};
+
+// A batch of independent tile tasks launched as one grid (grouped GEMM); passed by value
+// as a __grid_constant__ kernel parameter (16 * 88 + 68 bytes).
+constexpr int kMaxBatch = 16;
+struct TileBatch {
+    int n = 0;
+    int cta_start[kMaxBatch + 1] = {};
+    TileTask t[kMaxBatch];
+};
+
+// All tasks of a batch share transA / transB (dgemm_tile.cu).
+cudaError_t launch_dgemm_batch(bool ta, bool tb, TileBatch &b, cudaStream_t st);
+// Single task (batch of one).
 cudaError_t launch_dgemm_tile(bool ta, bool tb, int64_t M, int64_t N, int64_t K, double alpha,
                               const double *A, int64_t lda, const double *B, int64_t ldb,
                               double beta, double *C, int64_t ldc, cudaStream_t st);
