@@ -173,11 +173,24 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
     const int fr = lane >> 2, fc = lane & 3;
     const double *sAd = smem;
     const double *sBd = smem + STAGES * SA::kDoubles;
+    constexpr int KS = BK / 4;
+    // Fragments are double-buffered in registers: the loads for step ks+1 (or for step 0
+    // of the next k-block, right after the one barrier per block) are issued before the
+    // DMMAs of step ks, so shared-memory latency hides behind 32 DMMAs.
+    double fa[2][MF], fb[2][NF];
+    auto load_frags = [&](int buf, const double *a, const double *b, int ks) {
+#pragma unroll
+        for (int i = 0; i < MF; ++i) fa[buf][i] = a[SA::idx(wm + i * 8 + fr, ks * 4 + fc)];
+#pragma unroll
+        for (int j = 0; j < NF; ++j) fb[buf][j] = b[SB::idx(wn + j * 8 + fr, ks * 4 + fc)];
+    };
+    cp_wait<STAGES - 2>();
+    __syncthreads();
+    load_frags(0, sAd, sBd, 0);
 #pragma unroll 1
     for (int kb = 0; kb < KB; ++kb) {
-        cp_wait<STAGES - 2>();
-        __syncthreads();
         {
+            // stage (kb-1) % STAGES was released by the barrier of the previous block
             const int nk = kb + STAGES - 1;
             if (nk < KB) {
                 const int st = nk % STAGES;
@@ -191,16 +204,22 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
         const double *a = sAd + (kb % STAGES) * SA::kDoubles;
         const double *b = sBd + (kb % STAGES) * SB::kDoubles;
 #pragma unroll
-        for (int ks = 0; ks < BK; ks += 4) {
-            double fa[MF], fb[NF];
-#pragma unroll
-            for (int i = 0; i < MF; ++i) fa[i] = a[SA::idx(wm + i * 8 + fr, ks + fc)];
-#pragma unroll
-            for (int j = 0; j < NF; ++j) fb[j] = b[SB::idx(wn + j * 8 + fr, ks + fc)];
+        for (int ks = 0; ks < KS; ++ks) {
+            const int cur = ks & 1;
+            if (ks + 1 < KS) {
+                load_frags(cur ^ 1, a, b, ks + 1);
+            } else if (kb + 1 < KB) {
+                // next block's stage has landed for every thread; this block's stage is
+                // no longer read after this barrier
+                cp_wait<STAGES - 2>();
+                __syncthreads();
+                const int nx = (kb + 1) % STAGES;
+                load_frags(cur ^ 1, sAd + nx * SA::kDoubles, sBd + nx * SB::kDoubles, 0);
+            }
 #pragma unroll
             for (int i = 0; i < MF; ++i)
 #pragma unroll
-                for (int j = 0; j < NF; ++j) dmma(acc[i][j], fa[i], fb[j]);
+                for (int j = 0; j < NF; ++j) dmma(acc[i][j], fa[cur][i], fb[cur][j]);
         }
     }
     cp_wait<0>();
@@ -258,6 +277,9 @@ cudaError_t launch_cfg(TileBatch &b, cudaStream_t st) {
 //   1: 128x64  CTA, 4 warps of 64x32, BK 16, 4 stages, 2 CTAs/SM (independent barriers)
 //   2: 128x128 CTA, 8 warps of 64x32, BK 32, 3 stages
 //   4: 128x64  CTA, 4 warps of 64x32, BK 16, 3 stages, 2 CTAs/SM  (default)
+//   5: 128x64  CTA, 8 warps of 32x32, BK 16, 3 stages, 2 CTAs/SM (4 warps per scheduler)
+//   6: 64x128  CTA, 8 warps of 32x32, BK 16, 3 stages, 2 CTAs/SM
+//   7: 128x64  CTA, 8 warps of 32x32, BK 32, 2 stages, 2 CTAs/SM
 int g_kcfg = -1;
 int kcfg() {
     if (g_kcfg < 0) {
@@ -276,6 +298,12 @@ cudaError_t launch_t(TileBatch &b, cudaStream_t st) {
         return launch_cfg<128, 64, 64, 32, 16, 4, 2, TA, TB, VEC>(b, st);
     case 2:
         return launch_cfg<128, 128, 64, 32, 32, 3, 1, TA, TB, VEC>(b, st);
+    case 5:
+        return launch_cfg<128, 64, 32, 32, 16, 3, 2, TA, TB, VEC>(b, st);
+    case 6:
+        return launch_cfg<64, 128, 32, 32, 16, 3, 2, TA, TB, VEC>(b, st);
+    case 7:
+        return launch_cfg<128, 64, 32, 32, 32, 2, 2, TA, TB, VEC>(b, st);
     default:
         return launch_cfg<128, 64, 64, 32, 16, 3, 2, TA, TB, VEC>(b, st);
     }
