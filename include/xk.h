@@ -177,7 +177,8 @@ typedef struct xk_stats {
 } xk_stats_t;
 int xk_get_stats(xk_stats_t *out);
 int xk_reset_stats(void);
-/* 1 = time every tile kernel with CUDA events (bench roofline); 0 = off (default). */
+/* 1 = time every tile-kernel launch with CUDA events (bench roofline); grouped launches are
+ * then serialised on one kernel stream per GPU so each duration is its own.  0 = off. */
 int xk_set_kernel_timing(int on);
 
 /* (G+1) x (G+1) link matrix in MB/s, row = source, column = destination, index G =

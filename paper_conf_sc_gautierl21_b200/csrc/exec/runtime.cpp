@@ -94,7 +94,7 @@ int Runtime::init(const xk_config_t &cfg) {
     batch_count_.assign(G, 0);
     {
         const char *eb = std::getenv("XK_BATCH");
-        int mb = (eb && *eb) ? std::atoi(eb) : kMaxBatch;
+        int mb = (eb && *eb) ? std::atoi(eb) : 16;
         max_batch_ = std::max(1, std::min(kMaxBatch, mb));
     }
     // flags
@@ -463,7 +463,9 @@ int Runtime::flush_batch(int g) {
     int rc;
     if ((rc = set_dev(g))) return rc;
     const Device &d = devs_[g];
-    cudaStream_t s = d.ks[batch_count_[g]++ % cfg_.kstreams];
+    // kernel timing serialises the grouped launches on one stream so that each launch's
+    // event-timed duration is its own (no overlap with a concurrent launch)
+    cudaStream_t s = kernel_timing ? d.ks[0] : d.ks[batch_count_[g]++ % cfg_.kstreams];
     TileBatch tb;
     tb.n = (int)bt.recs.size();
     int64_t flops = 0;

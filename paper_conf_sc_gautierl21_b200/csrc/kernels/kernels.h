@@ -16,8 +16,8 @@ struct TileTask {
 };
 
 // A batch of independent tile tasks launched as one grid (grouped GEMM); passed by value
-// as a __grid_constant__ kernel parameter (16 * 88 + 68 bytes).
-constexpr int kMaxBatch = 16;
+// as a __grid_constant__ kernel parameter (32 * 88 + 136 bytes < 4 KB).
+constexpr int kMaxBatch = 32;
 struct TileBatch {
     int n = 0;
     int cta_start[kMaxBatch + 1] = {};
