@@ -206,6 +206,11 @@ int xk_get_topology(xk_topo_t *out);
 #define XK_SRC_HOST 3
 
 #define XK_ROUTINE_DGEMM 0
+#define XK_ROUTINE_DSYRK 1
+#define XK_ROUTINE_DSYR2K 2
+#define XK_ROUTINE_DSYMM 3
+#define XK_ROUTINE_DTRMM 4
+#define XK_ROUTINE_DTRSM 5
 #define XK_ROUTINE_COHERENT 100
 #define XK_ROUTINE_SYNC 101
 #define XK_ROUTINE_INVALIDATE 102
@@ -217,12 +222,21 @@ typedef struct xk_flags {
     int64_t tile;
 } xk_flags_t;
 
+/* Tile-task operations (TASK records, field op). */
+#define XK_OP_GEMM 0      /* C = alpha*op(A)*op(B) + beta*C */
+#define XK_OP_SCALE 1     /* C = beta*C (alpha == 0 or k == 0) */
+#define XK_OP_GEMM_TRI 2  /* GEMM on a diagonal tile writing only its uplo triangle (SYRK/SYR2K) */
+#define XK_OP_SYMM_DIAG 3 /* C = alpha*sym(A_ii)*B + beta*C or alpha*B*sym(A_jj) + beta*C */
+#define XK_OP_TRMM_DIAG 4 /* B = alpha*op(A_kk)*B or alpha*B*op(A_kk), in place */
+#define XK_OP_TRSM_DIAG 5 /* B = alpha*op(A_kk)^-1*B or alpha*B*op(A_kk)^-1, in place */
+
 /* One API call as seen by the planner.  Matrix addresses are identities only (never
- * dereferenced by the planner).  For XK_ROUTINE_COHERENT / INVALIDATE the view is
- * (m, n, C, ldc). */
+ * dereferenced by the planner).  The OUTPUT matrix is always (C, ldc): for TRMM/TRSM the
+ * BLAS "B" (m x n, updated in place) is passed as C.  transA doubles as SYRK/SYR2K's
+ * trans.  For XK_ROUTINE_COHERENT / INVALIDATE / PREFETCH the view is (m, n, C, ldc). */
 typedef struct xk_call {
     int routine;
-    char transA, transB;
+    char transA, transB, uplo, side, diag;
     int64_t m, n, k;
     double alpha, beta;
     uint64_t A, lda, B, ldb, C, ldc;
@@ -234,14 +248,17 @@ typedef struct xk_plan_rec {
     int32_t kind;      /* XK_REC_* */
     int32_t operand;   /* 0 = A, 1 = B, 2 = C of the call (coherent/prefetch: 2) */
     int64_t bi, bj;    /* tile coordinates in the STORED matrix (T x T grid at element 0,0) */
-    int64_t tk;        /* TASK: k-tile index (-1: scale-only task C <- beta*C) */
+    int64_t tk;        /* TASK: k-tile / step index of the tiled algorithm (-1: scale-only) */
     int64_t version;   /* tile version the record moves / produces */
     int32_t dst, src;  /* node ids: GPU 0..G-1 or XK_HOST */
     int32_t src_state; /* XK_SRC_* (copies); XK_SRC_NONE for tasks */
     int32_t depth;     /* forwarding depth of the destination copy (host = 0, H2D = 1) */
+    int32_t op;        /* TASK: XK_OP_*; copies: -1 */
+    int32_t reserved;
     int64_t t_start, t_end; /* virtual time, integer ns */
     int64_t work;      /* bytes (copies) or flops (tasks) */
-    int64_t dep[4];    /* seq of records this one waits on (-1 = none) */
+    int64_t dep[4];    /* seq of records this one waits on, one per task input in input order
+                          (copies: dep[0] = producer of the source copy); -1 = none */
 } xk_plan_rec_t;
 
 /* Planner sessions: the directory, clocks and link occupancy persist across calls

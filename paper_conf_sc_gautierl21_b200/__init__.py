@@ -211,10 +211,11 @@ def _flags(topo="ranked", optimistic=True, window=2, grid=(0, 0), tile=2048):
 
 
 def make_call(routine=ROUTINE_DGEMM, transA="N", transB="N", m=0, n=0, k=0, alpha=1.0, beta=0.0,
-              A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False):
+              A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False, uplo="L", side="L", diag="N"):
     c = _abi.Call()
     c.routine = routine
     c.transA, c.transB = _c(transA), _c(transB)
+    c.uplo, c.side, c.diag = _c(uplo), _c(side), _c(diag)
     c.m, c.n, c.k = m, n, k
     c.alpha, c.beta = alpha, beta
     c.A, c.lda, c.B, c.ldb, c.C, c.ldc = A, lda, B, ldb, C, ldc

@@ -21,7 +21,8 @@ XK_ERR_INTERNAL = 8
 TOPO_RANKED, TOPO_UNRANKED, TOPO_HOME = 0, 1, 2
 REC_H2D, REC_P2P, REC_TASK, REC_D2H = 0, 1, 2, 3
 SRC_NONE, SRC_VALID, SRC_INFLIGHT, SRC_HOST = 0, 1, 2, 3
-ROUTINE_DGEMM = 0
+ROUTINE_DGEMM, ROUTINE_DSYRK, ROUTINE_DSYR2K, ROUTINE_DSYMM, ROUTINE_DTRMM, ROUTINE_DTRSM = 0, 1, 2, 3, 4, 5
+OP_GEMM, OP_SCALE, OP_GEMM_TRI, OP_SYMM_DIAG, OP_TRMM_DIAG, OP_TRSM_DIAG = 0, 1, 2, 3, 4, 5
 ROUTINE_COHERENT, ROUTINE_SYNC, ROUTINE_INVALIDATE, ROUTINE_PREFETCH = 100, 101, 102, 103
 
 i64 = ctypes.c_int64
@@ -59,7 +60,8 @@ class Flags(ctypes.Structure):
 
 
 class Call(ctypes.Structure):
-    _fields_ = [("routine", c_int), ("transA", c_char), ("transB", c_char), ("m", i64), ("n", i64),
+    _fields_ = [("routine", c_int), ("transA", c_char), ("transB", c_char), ("uplo", c_char),
+                ("side", c_char), ("diag", c_char), ("m", i64), ("n", i64),
                 ("k", i64), ("alpha", c_double), ("beta", c_double), ("A", u64), ("lda", u64),
                 ("B", u64), ("ldb", u64), ("C", u64), ("ldc", u64), ("sync", c_int)]
 
@@ -68,16 +70,17 @@ class PlanRec(ctypes.Structure):
     _fields_ = [("seq", i64), ("kind", ctypes.c_int32), ("operand", ctypes.c_int32), ("bi", i64),
                 ("bj", i64), ("tk", i64), ("version", i64), ("dst", ctypes.c_int32),
                 ("src", ctypes.c_int32), ("src_state", ctypes.c_int32), ("depth", ctypes.c_int32),
+                ("op", ctypes.c_int32), ("reserved", ctypes.c_int32),
                 ("t_start", i64), ("t_end", i64), ("work", i64), ("dep", i64 * 4)]
 
     def as_tuple(self):
         return (self.seq, self.kind, self.operand, self.bi, self.bj, self.tk, self.version,
                 self.dst, self.src, self.src_state, self.depth, self.t_start, self.t_end,
-                self.work, tuple(self.dep))
+                self.work, tuple(self.dep), self.op)
 
 
 REC_FIELDS = ("seq", "kind", "operand", "bi", "bj", "tk", "version", "dst", "src", "src_state",
-              "depth", "t_start", "t_end", "work", "dep")
+              "depth", "t_start", "t_end", "work", "dep", "op")
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libxk.so")

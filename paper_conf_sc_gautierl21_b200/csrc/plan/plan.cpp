@@ -224,6 +224,7 @@ bool Planner::emit_copy(int key, int64_t ver, int d, int64_t treq, int operand,
     R.r.work = bytes;
     R.r.dep[0] = dep;
     R.r.dep[1] = R.r.dep[2] = R.r.dep[3] = -1;
+    R.r.op = -1;
     R.key = key;
     R.sub_rows = e.rows;
     R.sub_cols = e.cols;
@@ -264,6 +265,7 @@ void Planner::emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, i
     R.r.work = bytes;
     R.r.dep[0] = dep;
     R.r.dep[1] = R.r.dep[2] = R.r.dep[3] = -1;
+    R.r.op = -1;
     R.key = key;
     R.sub_r0 = r0;
     R.sub_c0 = c0;
@@ -279,28 +281,29 @@ void Planner::emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, i
     }
 }
 
-// steps 2, 3, 6, 7: per-GPU k-major lists in k-shifted anti-diagonal order, event loop
-// on the smallest request time, task timing, output versioning, D2H after last writer.
-int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double beta, char ta,
-                       char tb, std::vector<Rec> &out, std::string &err) {
+// steps 2, 3, 6, 7: per-GPU lists ordered by the generator's sort key (k-major, k-shifted
+// anti-diagonal), event loop on the smallest request time, task timing, output
+// versioning, D2H after the last writer of each output tile.
+int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &out, std::string &err) {
     const int G = topo_.G;
     const int W = std::max(1, flags_.window);
-    // pending reads per (key, version) in this call
+    // pending reads per (key, version) in this call; last writer per output tile
     std::map<std::pair<int, int64_t>, int64_t> readers;
-    for (auto &t : tasks)
-        for (auto &in : t.in) readers[{in.key, in.ver}]++;
+    std::map<int, size_t> last;
+    for (size_t q = 0; q < tasks.size(); ++q) {
+        for (auto &in : tasks[q].in) readers[{in.key, in.ver}]++;
+        auto it = last.find(tasks[q].out_key);
+        if (it == last.end() || tasks[it->second].out_ver < tasks[q].out_ver) last[tasks[q].out_key] = q;
+    }
+    for (auto &kv : last) tasks[kv.second].last_writer = true;
     std::vector<std::vector<int>> lists(G);
-    int64_t tmax = 1;
-    for (auto &t : tasks) tmax = std::max(tmax, std::max(t.i, t.j) + 1);
     for (size_t q = 0; q < tasks.size(); ++q) lists[tasks[q].gpu].push_back((int)q);
     for (int d = 0; d < G; ++d) {
         std::stable_sort(lists[d].begin(), lists[d].end(), [&](int a, int b) {
             const Task &x = tasks[a], &y = tasks[b];
-            int64_t kx = std::max<int64_t>(x.tk, 0), ky = std::max<int64_t>(y.tk, 0);
-            auto key = [&](const Task &t, int64_t k) {
-                return std::make_tuple(k, (t.i + t.j + k) % tmax, t.i, t.j);
-            };
-            return key(x, kx) < key(y, ky);
+            for (int q = 0; q < 5; ++q)
+                if (x.skey[q] != y.skey[q]) return x.skey[q] < y.skey[q];
+            return false;
         });
     }
     std::vector<size_t> pos(G, 0);
@@ -336,7 +339,8 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double
         const int64_t treq = best_treq;
         int64_t in_ready = 0;
         int64_t deps[4] = {-1, -1, -1, -1};
-        for (auto &in : t.in) {
+        for (size_t p = 0; p < t.in.size(); ++p) {
+            const Input &in = t.in[p];
             Entry &e = entries_[in.key];
             if (!(e.gpu[d].present && e.gpu[d].ver == in.ver) &&
                 !emit_copy(in.key, in.ver, d, treq, in.operand, out)) {
@@ -344,7 +348,7 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double
                 return XK_ERR_INTERNAL;
             }
             in_ready = std::max(in_ready, e.gpu[d].t_done);
-            deps[in.operand] = e.gpu[d].producer;
+            if (p < 4) deps[p] = e.gpu[d].producer;
             readers[{in.key, in.ver}]--;
         }
         int64_t t0 = std::max(gpu_free_[d], in_ready);
@@ -365,18 +369,23 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double
         R.r.src = d;
         R.r.src_state = XK_SRC_NONE;
         R.r.depth = 0;
+        R.r.op = t.op;
         R.r.t_start = t0;
         R.r.t_end = t1;
         R.r.work = t.flops;
         for (int q = 0; q < 4; ++q) R.r.dep[q] = deps[q];
         R.key = t.out_key;
+        R.op = t.op;
         R.keyA = t.keyA;
         R.keyB = t.keyB;
-        R.ta = ta;
-        R.tb = tb;
-        R.alpha = alpha;
-        // beta applies on the first task of the chain only (k == 0 or scale-only)
-        R.beta = (t.tk <= 0) ? beta : 1.0;
+        R.ta = t.ta;
+        R.tb = t.tb;
+        R.side = t.side;
+        R.uplo = t.uplo;
+        R.diag = t.diag;
+        R.tri = t.tri;
+        R.alpha = t.alpha;
+        R.beta = t.beta;
         R.m = t.m;
         R.n = t.n;
         R.k = t.k;
@@ -397,10 +406,13 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double
     return XK_OK;
 }
 
+static bool is_t(char c) { return c == 'T' || c == 't' || c == 'C' || c == 'c'; }
+static char up(char c) { return (c >= 'a' && c <= 'z') ? (char)(c - 32) : c; }
+
+// DGEMM (PLASMA pdgemm structure): C(i,j) k-chains, beta on the first task.
 int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
     const int64_t m = c.m, n = c.n, k = c.k, T = flags_.T;
-    const bool ta = c.transA == 'T' || c.transA == 't' || c.transA == 'C' || c.transA == 'c';
-    const bool tb = c.transB == 'T' || c.transB == 't' || c.transB == 'C' || c.transB == 'c';
+    const bool ta = is_t(c.transA), tb = is_t(c.transB);
     if (m == 0 || n == 0 || ((c.alpha == 0.0 || k == 0) && c.beta == 1.0)) return XK_OK;
     const bool scale_only = (c.alpha == 0.0 || k == 0);
     int mc = find_or_add_matrix(c.C, (int64_t)c.ldc, m, n, err);
@@ -413,23 +425,28 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
         if (mb < 0) return XK_ERR_UNSUPPORTED;
     }
     const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
+    const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
+    Versions V;
+    V.e = &entries_;
     std::vector<Task> tasks;
     for (int64_t j = 0; j < tn; ++j) {
         for (int64_t i = 0; i < tm; ++i) {
             int keyC = key_of(mc, i, j);
-            int64_t v0 = entries_[keyC].ver;
             int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
             if (scale_only) {
                 Task t;
                 t.gpu = owner(i, j);
+                t.op = XK_OP_SCALE;
                 t.out_key = keyC;
-                t.out_ver = v0 + 1;
-                if (c.beta != 0.0) t.in.push_back({keyC, v0, 2});
+                if (c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                t.out_ver = V.bump(keyC);
+                t.beta = c.beta;
                 t.tk = -1;
                 t.i = i; t.j = j;
                 t.m = mt; t.n = nt; t.k = 0;
                 t.flops = mt * nt;
-                t.last_writer = true;
+                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
+                std::copy(sk, sk + 5, t.skey);
                 tasks.push_back(t);
                 continue;
             }
@@ -439,24 +456,363 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                 int keyB = tb ? key_of(mb, j, kk) : key_of(mb, kk, j);
                 Task t;
                 t.gpu = owner(i, j);
+                t.op = XK_OP_GEMM;
                 t.out_key = keyC;
-                t.out_ver = v0 + kk + 1;
-                t.in.push_back({keyA, entries_[keyA].ver, 0});
-                t.in.push_back({keyB, entries_[keyB].ver, 1});
-                if (kk > 0) t.in.push_back({keyC, v0 + kk, 2});
-                else if (c.beta != 0.0) t.in.push_back({keyC, v0, 2});
+                t.in.push_back({keyA, V.get(keyA), 0});
+                t.in.push_back({keyB, V.get(keyB), 1});
+                if (kk > 0 || c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                t.out_ver = V.bump(keyC);
+                t.keyA = keyA;
+                t.keyB = keyB;
+                t.ta = ta ? 'T' : 'N';
+                t.tb = tb ? 'T' : 'N';
+                t.alpha = c.alpha;
+                t.beta = (kk == 0) ? c.beta : 1.0;
                 t.tk = kk;
                 t.i = i; t.j = j;
                 t.m = mt; t.n = nt; t.k = kt;
                 t.flops = 2 * mt * nt * kt;
-                t.last_writer = (kk == tkn - 1);
-                t.keyA = keyA;
-                t.keyB = keyB;
+                int64_t sk[5] = {kk, (i + j + kk) % tmod, i, j, 0};
+                std::copy(sk, sk + 5, t.skey);
                 tasks.push_back(t);
             }
         }
     }
-    return run_tasks(tasks, c.sync != 0, c.alpha, c.beta, ta ? 'T' : 'N', tb ? 'T' : 'N', out, err);
+    return run_tasks(tasks, c.sync != 0, out, err);
+}
+
+// DSYRK / DSYR2K (PLASMA pdsyrk / pdsyr2k): tiles of the uplo triangle of C; off-diagonal
+// tiles are GEMM k-chains, diagonal tiles GEMM_TRI tasks writing only the triangle.  A
+// diagonal tile is always copied in (even when beta == 0) so the untouched triangle goes
+// back to the host bit for bit (BLAS: it is not referenced).
+int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std::string &err) {
+    const int64_t n = c.n, k = c.k, T = flags_.T;
+    const bool tr = is_t(c.transA), lower = up(c.uplo) == 'L';
+    if (n == 0 || ((c.alpha == 0.0 || k == 0) && c.beta == 1.0)) return XK_OK;
+    const bool scale_only = (c.alpha == 0.0 || k == 0);
+    int mc = find_or_add_matrix(c.C, (int64_t)c.ldc, n, n, err);
+    if (mc < 0) return XK_ERR_UNSUPPORTED;
+    int ma = -1, mb = -1;
+    if (!scale_only) {
+        ma = find_or_add_matrix(c.A, (int64_t)c.lda, tr ? k : n, tr ? n : k, err);
+        if (ma < 0) return XK_ERR_UNSUPPORTED;
+        if (two) {
+            mb = find_or_add_matrix(c.B, (int64_t)c.ldb, tr ? k : n, tr ? n : k, err);
+            if (mb < 0) return XK_ERR_UNSUPPORTED;
+        }
+    }
+    const int64_t tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
+    const int64_t tmod = std::max<int64_t>(1, tn);
+    const int tri = lower ? 1 : 2;
+    Versions V;
+    V.e = &entries_;
+    std::vector<Task> tasks;
+    auto opnd = [&](int mat, int64_t r, int64_t l) {  // tile (r, l) of op(X), X n x k
+        return tr ? key_of(mat, l, r) : key_of(mat, r, l);
+    };
+    for (int64_t j = 0; j < tn; ++j) {
+        for (int64_t i = 0; i < tn; ++i) {
+            if (lower ? (i < j) : (i > j)) continue;
+            const bool dg = (i == j);
+            int keyC = key_of(mc, i, j);
+            int64_t mt = std::min(T, n - i * T), nt = std::min(T, n - j * T);
+            if (scale_only) {
+                Task t;
+                t.gpu = owner(i, j);
+                t.op = XK_OP_SCALE;
+                t.tri = dg ? tri : 0;
+                t.out_key = keyC;
+                if (c.beta != 0.0 || dg) t.in.push_back({keyC, V.get(keyC), 2});
+                t.out_ver = V.bump(keyC);
+                t.beta = c.beta;
+                t.tk = -1;
+                t.i = i; t.j = j;
+                t.m = mt; t.n = nt;
+                t.flops = mt * nt;
+                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
+                std::copy(sk, sk + 5, t.skey);
+                tasks.push_back(t);
+                continue;
+            }
+            bool first = true;
+            for (int64_t l = 0; l < tkn; ++l) {
+                int64_t kt = std::min(T, k - l * T);
+                for (int s = 0; s < (two ? 2 : 1); ++s) {
+                    // SYRK: op(A)_i op(A)_j^T.  SYR2K: s=0 op(A)_i op(B)_j^T, s=1 op(B)_i op(A)_j^T
+                    int xa = (two && s == 1) ? mb : ma, xb = (two && s == 0) ? mb : ma;
+                    int keyA = opnd(xa, i, l), keyB = opnd(xb, j, l);
+                    Task t;
+                    t.gpu = owner(i, j);
+                    t.op = dg ? XK_OP_GEMM_TRI : XK_OP_GEMM;
+                    t.tri = dg ? tri : 0;
+                    t.out_key = keyC;
+                    t.in.push_back({keyA, V.get(keyA), xa == ma ? 0 : 1});
+                    t.in.push_back({keyB, V.get(keyB), xb == ma ? 0 : 1});
+                    if (!first || c.beta != 0.0 || dg) t.in.push_back({keyC, V.get(keyC), 2});
+                    t.out_ver = V.bump(keyC);
+                    t.keyA = keyA;
+                    t.keyB = keyB;
+                    t.ta = tr ? 'T' : 'N';  // op(A) tile = X(i,l) or X(l,i)^T
+                    t.tb = tr ? 'N' : 'T';  // op(B) tile = X(j,l)^T or X(l,j)
+                    t.alpha = c.alpha;
+                    t.beta = first ? c.beta : 1.0;
+                    t.tk = l;
+                    t.i = i; t.j = j;
+                    t.m = mt; t.n = nt; t.k = kt;
+                    t.flops = dg ? kt * nt * (nt + 1) : 2 * mt * nt * kt;
+                    int64_t sk[5] = {2 * l + s, (i + j + l) % tmod, i, j, 0};
+                    std::copy(sk, sk + 5, t.skey);
+                    tasks.push_back(t);
+                    first = false;
+                }
+            }
+        }
+    }
+    return run_tasks(tasks, c.sync != 0, out, err);
+}
+
+// DSYMM (PLASMA pdsymm): C(i,j) k-chains over sym(A); the diagonal tile of A is used
+// symmetrically expanded from its uplo triangle (SYMM_DIAG), off-diagonal tiles are read
+// from the uplo triangle, transposed when they lie in the other one.
+int Planner::plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
+    const int64_t m = c.m, n = c.n, T = flags_.T;
+    const bool left = up(c.side) == 'L', lower = up(c.uplo) == 'L';
+    if (m == 0 || n == 0 || (c.alpha == 0.0 && c.beta == 1.0)) return XK_OK;
+    const bool scale_only = (c.alpha == 0.0);
+    const int64_t ka = left ? m : n;
+    int mc = find_or_add_matrix(c.C, (int64_t)c.ldc, m, n, err);
+    if (mc < 0) return XK_ERR_UNSUPPORTED;
+    int ma = -1, mb = -1;
+    if (!scale_only) {
+        ma = find_or_add_matrix(c.A, (int64_t)c.lda, ka, ka, err);
+        if (ma < 0) return XK_ERR_UNSUPPORTED;
+        mb = find_or_add_matrix(c.B, (int64_t)c.ldb, m, n, err);
+        if (mb < 0) return XK_ERR_UNSUPPORTED;
+    }
+    const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tl = cdiv(ka, T);
+    const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
+    Versions V;
+    V.e = &entries_;
+    std::vector<Task> tasks;
+    for (int64_t j = 0; j < tn; ++j) {
+        for (int64_t i = 0; i < tm; ++i) {
+            int keyC = key_of(mc, i, j);
+            int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
+            if (scale_only) {
+                Task t;
+                t.gpu = owner(i, j);
+                t.op = XK_OP_SCALE;
+                t.out_key = keyC;
+                if (c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                t.out_ver = V.bump(keyC);
+                t.beta = c.beta;
+                t.tk = -1;
+                t.i = i; t.j = j;
+                t.m = mt; t.n = nt;
+                t.flops = mt * nt;
+                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
+                std::copy(sk, sk + 5, t.skey);
+                tasks.push_back(t);
+                continue;
+            }
+            for (int64_t l = 0; l < tl; ++l) {
+                int64_t kt = std::min(T, ka - l * T);
+                // sym(A) tile (r, q): stored (r, q) if it lies in the uplo triangle, else (q, r)^T
+                int64_t r = left ? i : l, q = left ? l : j;
+                bool in_tri = lower ? (r >= q) : (r <= q);
+                int keyAt = in_tri ? key_of(ma, r, q) : key_of(ma, q, r);
+                int keyBt = left ? key_of(mb, l, j) : key_of(mb, i, l);
+                Task t;
+                t.gpu = owner(i, j);
+                t.out_key = keyC;
+                t.side = left ? 'L' : 'R';
+                t.uplo = lower ? 'L' : 'U';
+                if (r == q) {
+                    t.op = XK_OP_SYMM_DIAG;
+                    t.keyA = keyAt;
+                    t.keyB = keyBt;
+                    t.in.push_back({keyAt, V.get(keyAt), 0});
+                    t.in.push_back({keyBt, V.get(keyBt), 1});
+                } else if (left) {
+                    t.op = XK_OP_GEMM;
+                    t.keyA = keyAt;
+                    t.keyB = keyBt;
+                    t.ta = in_tri ? 'N' : 'T';
+                    t.tb = 'N';
+                    t.in.push_back({keyAt, V.get(keyAt), 0});
+                    t.in.push_back({keyBt, V.get(keyBt), 1});
+                } else {
+                    t.op = XK_OP_GEMM;  // C(i,j) += B(i,l) * sym(A)(l,j)
+                    t.keyA = keyBt;
+                    t.keyB = keyAt;
+                    t.ta = 'N';
+                    t.tb = in_tri ? 'N' : 'T';
+                    t.in.push_back({keyBt, V.get(keyBt), 1});
+                    t.in.push_back({keyAt, V.get(keyAt), 0});
+                }
+                if (l > 0 || c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                t.out_ver = V.bump(keyC);
+                t.alpha = c.alpha;
+                t.beta = (l == 0) ? c.beta : 1.0;
+                t.tk = l;
+                t.i = i; t.j = j;
+                t.m = mt; t.n = nt; t.k = kt;
+                t.flops = 2 * mt * nt * kt;
+                int64_t sk[5] = {l, (i + j + l) % tmod, i, j, 0};
+                std::copy(sk, sk + 5, t.skey);
+                tasks.push_back(t);
+            }
+        }
+    }
+    return run_tasks(tasks, c.sync != 0, out, err);
+}
+
+// DTRMM / DTRSM (PLASMA pdtrmm / pdtrsm) on the output B (passed as C).  op(A) is
+// effectively lower iff (uplo == 'L') != (transA == 'T').  TRSM walks k in the solve
+// direction: diagonal solve of row (col) k, then GEMM updates of the remaining rows (cols)
+// with the solved tiles -- GPU-produced tiles are read by peers (the topology heuristic's
+// native case inside one call).  TRMM walks rows (cols) so that every GEMM reads tiles of
+// B that are still unmodified (WAR on the in-place update is enforced by the planner).
+int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, std::string &err) {
+    const int64_t m = c.m, n = c.n, T = flags_.T;
+    const bool left = up(c.side) == 'L', lower = up(c.uplo) == 'L', tr = is_t(c.transA);
+    const bool elow = (lower != tr);
+    if (m == 0 || n == 0) return XK_OK;
+    const int64_t ka = left ? m : n;
+    int mc = find_or_add_matrix(c.C, (int64_t)c.ldc, m, n, err);
+    if (mc < 0) return XK_ERR_UNSUPPORTED;
+    const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tk = cdiv(ka, T);
+    const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
+    Versions V;
+    V.e = &entries_;
+    std::vector<Task> tasks;
+    if (c.alpha == 0.0) {  // B <- 0, A not referenced
+        for (int64_t j = 0; j < tn; ++j)
+            for (int64_t i = 0; i < tm; ++i) {
+                int keyC = key_of(mc, i, j);
+                Task t;
+                t.gpu = owner(i, j);
+                t.op = XK_OP_SCALE;
+                t.out_key = keyC;
+                t.out_ver = V.bump(keyC);
+                t.beta = 0.0;
+                t.tk = -1;
+                t.i = i; t.j = j;
+                t.m = std::min(T, m - i * T);
+                t.n = std::min(T, n - j * T);
+                t.flops = t.m * t.n;
+                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
+                std::copy(sk, sk + 5, t.skey);
+                tasks.push_back(t);
+            }
+        return run_tasks(tasks, c.sync != 0, out, err);
+    }
+    int ma = find_or_add_matrix(c.A, (int64_t)c.lda, ka, ka, err);
+    if (ma < 0) return XK_ERR_UNSUPPORTED;
+    auto opA = [&](int64_t r, int64_t q) { return tr ? key_of(ma, q, r) : key_of(ma, r, q); };
+    const char tA = tr ? 'T' : 'N';
+    // k order: forward when (left & lower) or (right & upper) for TRSM; TRMM the reverse
+    const bool fwd = solve ? (left == elow) : (left != elow);
+    const int64_t nsteps = tk;
+    const int64_t other = left ? tn : tm;  // tiles along the untouched dimension
+    for (int64_t s = 0; s < nsteps; ++s) {
+        const int64_t kx = fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
+        const double a_s = solve ? ((s == 0) ? c.alpha : 1.0) : c.alpha;
+        for (int64_t o = 0; o < other; ++o) {
+            const int64_t bi = left ? kx : o, bj = left ? o : kx;
+            int keyD = opA(kx, kx), keyO = key_of(mc, bi, bj);
+            const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
+            // diagonal task on B(kx, o) (left) / B(o, kx) (right)
+            Task t;
+            t.gpu = owner(bi, bj);
+            t.op = solve ? XK_OP_TRSM_DIAG : XK_OP_TRMM_DIAG;
+            t.out_key = keyO;
+            t.keyA = keyD;
+            t.in.push_back({keyD, V.get(keyD), 0});
+            t.in.push_back({keyO, V.get(keyO), 2});
+            t.out_ver = V.bump(keyO);
+            t.ta = tA;
+            t.side = left ? 'L' : 'R';
+            t.uplo = lower ? 'L' : 'U';
+            t.diag = up(c.diag);
+            t.alpha = a_s;
+            t.tk = s;
+            t.i = bi; t.j = bj;
+            t.m = mt; t.n = nt; t.k = left ? mt : nt;
+            t.flops = left ? mt * mt * nt : mt * nt * nt;
+            int64_t sk[5] = {s, 0, (bi + bj + s) % tmod, bi, bj};
+            std::copy(sk, sk + 5, t.skey);
+            tasks.push_back(t);
+            // TRMM: this tile's remaining contributions (sources still unmodified)
+            if (!solve) {
+                int64_t ph = 1;
+                for (int64_t q = 0; q < tk; ++q) {
+                    const bool contributes = left ? (elow ? q < kx : q > kx) : (elow ? q > kx : q < kx);
+                    if (!contributes) continue;
+                    int keyA_ = left ? opA(kx, q) : key_of(mc, bi, q);
+                    int keyB_ = left ? key_of(mc, q, bj) : opA(q, kx);
+                    const int64_t kt = std::min(T, ka - q * T);
+                    Task g;
+                    g.gpu = owner(bi, bj);
+                    g.op = XK_OP_GEMM;
+                    g.out_key = keyO;
+                    g.keyA = keyA_;
+                    g.keyB = keyB_;
+                    g.ta = left ? tA : 'N';
+                    g.tb = left ? 'N' : tA;
+                    g.in.push_back({keyA_, V.get(keyA_), left ? 0 : 2});
+                    g.in.push_back({keyB_, V.get(keyB_), left ? 2 : 0});
+                    g.in.push_back({keyO, V.get(keyO), 2});
+                    g.out_ver = V.bump(keyO);
+                    g.alpha = c.alpha;
+                    g.beta = 1.0;
+                    g.tk = s;
+                    g.i = bi; g.j = bj;
+                    g.m = mt; g.n = nt; g.k = kt;
+                    g.flops = 2 * mt * nt * kt;
+                    int64_t sk2[5] = {s, ph++, (bi + bj + s) % tmod, bi, bj};
+                    std::copy(sk2, sk2 + 5, g.skey);
+                    tasks.push_back(g);
+                }
+            }
+        }
+        if (!solve) continue;
+        // TRSM: update the rows (cols) still to be solved with the solved tiles of step s
+        for (int64_t r = 0; r < tk; ++r) {
+            const bool later = fwd ? r > kx : r < kx;
+            if (!later) continue;
+            for (int64_t o = 0; o < other; ++o) {
+                const int64_t bi = left ? r : o, bj = left ? o : r;
+                int keyO = key_of(mc, bi, bj);
+                int keyA_ = left ? opA(r, kx) : key_of(mc, bi, kx);
+                int keyB_ = left ? key_of(mc, kx, bj) : opA(kx, r);
+                const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
+                const int64_t kt = std::min(T, ka - kx * T);
+                Task g;
+                g.gpu = owner(bi, bj);
+                g.op = XK_OP_GEMM;
+                g.out_key = keyO;
+                g.keyA = keyA_;
+                g.keyB = keyB_;
+                g.ta = left ? tA : 'N';
+                g.tb = left ? 'N' : tA;
+                g.in.push_back({keyA_, V.get(keyA_), left ? 0 : 2});
+                g.in.push_back({keyB_, V.get(keyB_), left ? 2 : 0});
+                g.in.push_back({keyO, V.get(keyO), 2});
+                g.out_ver = V.bump(keyO);
+                g.alpha = -1.0;
+                g.beta = a_s;
+                g.tk = s;
+                g.i = bi; g.j = bj;
+                g.m = mt; g.n = nt; g.k = kt;
+                g.flops = 2 * mt * nt * kt;
+                int64_t sk[5] = {s, 1, (bi + bj + s) % tmod, bi, bj};
+                std::copy(sk, sk + 5, g.skey);
+                tasks.push_back(g);
+            }
+        }
+    }
+    return run_tasks(tasks, c.sync != 0, out, err);
 }
 
 bool Planner::view_tiles(uint64_t base, int64_t m, int64_t n, int64_t ld, int *mat, int64_t *r0,
@@ -567,25 +923,66 @@ void Planner::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
     }
 }
 
-int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
+// After a synchronous routine: a full sync point, then the operands' device copies are
+// dropped (sync routines are drop-in).
+void Planner::finish_call(const xk_call_t &c) {
+    full_sync();
+    const bool ta = is_t(c.transA), tb = is_t(c.transB);
+    const bool left = up(c.side) == 'L';
     switch (c.routine) {
-    case XK_ROUTINE_DGEMM: {
-        int rc = plan_gemm(c, out, err);
-        if (rc) return rc;
-        if (c.sync) {
-            // the library waits here; then a full sync point and invalidation of the
-            // operands' device copies (sync routines are drop-in)
-            full_sync();
-            const bool ta = c.transA == 'T' || c.transA == 't' || c.transA == 'C' || c.transA == 'c';
-            const bool tb = c.transB == 'T' || c.transB == 't' || c.transB == 'C' || c.transB == 'c';
-            if (c.alpha != 0.0 && c.k > 0) {
-                invalidate(c.A, ta ? c.k : c.m, ta ? c.m : c.k, (int64_t)c.lda);
-                invalidate(c.B, tb ? c.n : c.k, tb ? c.k : c.n, (int64_t)c.ldb);
-            }
-            invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+    case XK_ROUTINE_DGEMM:
+        if (c.alpha != 0.0 && c.k > 0) {
+            invalidate(c.A, ta ? c.k : c.m, ta ? c.m : c.k, (int64_t)c.lda);
+            invalidate(c.B, tb ? c.n : c.k, tb ? c.k : c.n, (int64_t)c.ldb);
         }
-        return XK_OK;
+        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        break;
+    case XK_ROUTINE_DSYRK:
+    case XK_ROUTINE_DSYR2K:
+        if (c.alpha != 0.0 && c.k > 0) {
+            invalidate(c.A, ta ? c.k : c.n, ta ? c.n : c.k, (int64_t)c.lda);
+            if (c.routine == XK_ROUTINE_DSYR2K)
+                invalidate(c.B, ta ? c.k : c.n, ta ? c.n : c.k, (int64_t)c.ldb);
+        }
+        invalidate(c.C, c.n, c.n, (int64_t)c.ldc);
+        break;
+    case XK_ROUTINE_DSYMM:
+        if (c.alpha != 0.0) {
+            const int64_t ka = left ? c.m : c.n;
+            invalidate(c.A, ka, ka, (int64_t)c.lda);
+            invalidate(c.B, c.m, c.n, (int64_t)c.ldb);
+        }
+        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        break;
+    default: {  // TRMM / TRSM
+        const int64_t ka = left ? c.m : c.n;
+        if (c.alpha != 0.0) invalidate(c.A, ka, ka, (int64_t)c.lda);
+        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
     }
+    }
+}
+
+int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
+    int rc;
+    switch (c.routine) {
+    case XK_ROUTINE_DGEMM:
+        rc = plan_gemm(c, out, err);
+        break;
+    case XK_ROUTINE_DSYRK:
+        rc = plan_syrk(c, false, out, err);
+        break;
+    case XK_ROUTINE_DSYR2K:
+        rc = plan_syrk(c, true, out, err);
+        break;
+    case XK_ROUTINE_DSYMM:
+        rc = plan_symm(c, out, err);
+        break;
+    case XK_ROUTINE_DTRMM:
+        rc = plan_trxm(c, false, out, err);
+        break;
+    case XK_ROUTINE_DTRSM:
+        rc = plan_trxm(c, true, out, err);
+        break;
     case XK_ROUTINE_COHERENT:
         return plan_coherent(c, out, err, false);
     case XK_ROUTINE_SYNC:
@@ -600,6 +997,25 @@ int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
         err = "unknown routine";
         return XK_ERR_CONFIG;
     }
+    if (rc) return rc;
+    // a quick return (BLAS: nothing to do) is not a synchronisation point
+    bool quick;
+    switch (c.routine) {
+    case XK_ROUTINE_DGEMM:
+        quick = c.m == 0 || c.n == 0 || ((c.alpha == 0.0 || c.k == 0) && c.beta == 1.0);
+        break;
+    case XK_ROUTINE_DSYRK:
+    case XK_ROUTINE_DSYR2K:
+        quick = c.n == 0 || ((c.alpha == 0.0 || c.k == 0) && c.beta == 1.0);
+        break;
+    case XK_ROUTINE_DSYMM:
+        quick = c.m == 0 || c.n == 0 || (c.alpha == 0.0 && c.beta == 1.0);
+        break;
+    default:
+        quick = c.m == 0 || c.n == 0;
+    }
+    if (c.sync && !quick) finish_call(c);
+    return XK_OK;
 }
 
 }  // namespace xk

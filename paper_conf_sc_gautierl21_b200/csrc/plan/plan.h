@@ -63,10 +63,13 @@ struct Rec {
     int key = -1;                 // directory entry id
     int64_t sub_r0 = 0, sub_c0 = 0, sub_rows = 0, sub_cols = 0;  // D2H intersection (tile-relative)
     // task description (TASK records)
+    int op = XK_OP_GEMM;
     char ta = 'N', tb = 'N';
+    char side = 'L', uplo = 'L', diag = 'N';  // diagonal-tile ops
+    int tri = 0;                  // GEMM_TRI / SCALE on a diagonal tile: 1 lower, 2 upper
     double alpha = 1.0, beta = 0.0;
-    int keyA = -1, keyB = -1;     // input tiles on dst (-1: none)
-    int64_t m = 0, n = 0, k = 0;  // task shape
+    int keyA = -1, keyB = -1;     // tiles in the kernel's A and B roles on dst (-1: none)
+    int64_t m = 0, n = 0, k = 0;  // task shape (output rows, cols, inner / triangle order)
 };
 
 class Planner {
@@ -94,16 +97,28 @@ public:
 private:
     struct Input { int key; int64_t ver; int operand; };
     struct Task {
-        int gpu;
-        int out_key;
-        int64_t out_ver;            // version produced
-        std::vector<Input> in;      // in operand order A, B, C
-        int64_t tk;                 // k index, -1 scale-only
-        int64_t i, j;               // output tile coords (op space)
-        int64_t m, n, k;            // shape
-        int64_t flops;
-        bool last_writer;           // last write of out_key in this call
-        int keyA = -1, keyB = -1;
+        int gpu = 0;
+        int op = XK_OP_GEMM;
+        int out_key = -1;
+        int64_t out_ver = 0;        // version produced
+        std::vector<Input> in;      // inputs in position order (deps follow this order)
+        int keyA = -1, keyB = -1;   // kernel roles
+        char ta = 'N', tb = 'N', side = 'L', uplo = 'L', diag = 'N';
+        int tri = 0;
+        double alpha = 1.0, beta = 0.0;
+        int64_t tk = 0;             // step index (-1 scale-only)
+        int64_t i = 0, j = 0;       // output tile coords
+        int64_t m = 0, n = 0, k = 0;
+        int64_t flops = 0;
+        bool last_writer = false;   // last write of out_key in this call
+        int64_t skey[5] = {0, 0, 0, 0, 0};  // per-GPU list order
+    };
+    // symbolic versions while a call's task list is generated (program order)
+    struct Versions {
+        std::unordered_map<int, int64_t> cur;
+        const std::vector<Entry> *e = nullptr;
+        int64_t get(int key) { auto it = cur.find(key); return it == cur.end() ? (*e)[key].ver : it->second; }
+        int64_t bump(int key) { int64_t v = get(key) + 1; cur[key] = v; return v; }
     };
 
     int find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t cols, std::string &err);
@@ -114,9 +129,12 @@ private:
     void emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, int64_t cols,
                   int64_t ready, int64_t dep, int operand, std::vector<Rec> &out);
     int plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
+    int plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std::string &err);
+    int plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
+    int plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, std::string &err);
+    void finish_call(const xk_call_t &c);
     int plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::string &err, bool prefetch);
-    int run_tasks(std::vector<Task> &tasks, bool sync, double alpha, double beta, char ta,
-                  char tb, std::vector<Rec> &out, std::string &err);
+    int run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &out, std::string &err);
     bool view_tiles(uint64_t base, int64_t m, int64_t n, int64_t ld, int *mat,
                     int64_t *r0, int64_t *c0) const;
 

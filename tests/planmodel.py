@@ -20,7 +20,9 @@ H2D, P2P, TASK, D2H = 0, 1, 2, 3
 S_NONE, S_VALID, S_INFLIGHT, S_HOST = 0, 1, 2, 3
 RANKED, UNRANKED, HOME = 0, 1, 2
 HOSTID = -1
-DGEMM, COHERENT, SYNC, INVALIDATE, PREFETCH = 0, 100, 101, 102, 103
+DGEMM, DSYRK, DSYR2K, DSYMM, DTRMM, DTRSM = 0, 1, 2, 3, 4, 5
+COHERENT, SYNC, INVALIDATE, PREFETCH = 100, 101, 102, 103
+OP_GEMM, OP_SCALE, OP_GEMM_TRI, OP_SYMM_DIAG, OP_TRMM_DIAG, OP_TRSM_DIAG = 0, 1, 2, 3, 4, 5
 
 
 def ceil_div(a, b):
@@ -140,7 +142,7 @@ class Model:
         end = start + self.nsec(nbytes, self.bw[self.idx(src)][d])
         self.link[lk] = end
         out.append((self.seq, H2D if src == HOSTID else P2P, operand, t.bi, t.bj, -1, ver, d, src,
-                    state, depth, start, end, nbytes, (dep, -1, -1, -1)))
+                    state, depth, start, end, nbytes, (dep, -1, -1, -1), -1))
         t.gpus[d] = Copy(ver, end, self.seq, depth)
         self.seq += 1
 
@@ -152,25 +154,52 @@ class Model:
         end = start + self.nsec(nbytes, self.bw[src][self.G])
         self.link[lk] = end
         out.append((self.seq, D2H, 2, t.bi, t.bj, -1, t.ver, HOSTID, src, S_VALID, 0, start, end,
-                    nbytes, (dep, -1, -1, -1)))
+                    nbytes, (dep, -1, -1, -1), -1))
         if (r0, c0, rows, cols) == (0, 0, t.rows, t.cols):
             t.host = Copy(t.ver, end, self.seq, 0)
         self.seq += 1
 
     # ------------------------------------------------------------------ calls
     def call(self, routine=DGEMM, transA="N", transB="N", m=0, n=0, k=0, alpha=1.0, beta=0.0,
-             A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False):
+             A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False, uplo="L", side="L", diag="N"):
         out = []
-        if routine == DGEMM:
-            self.gemm(transA.upper() in "TC", transB.upper() in "TC", m, n, k, alpha, beta,
-                      A, lda, B, ldb, C, ldc, sync, out)
-            if sync:
+        ta, tb = transA.upper() in "TC", transB.upper() in "TC"
+        lower, left = uplo.upper() == "L", side.upper() == "L"
+        if routine in (DGEMM, DSYRK, DSYR2K, DSYMM, DTRMM, DTRSM):
+            if routine == DGEMM:
+                tasks = self.gen_gemm(ta, tb, m, n, k, alpha, beta, A, lda, B, ldb, C, ldc)
+            elif routine in (DSYRK, DSYR2K):
+                tasks = self.gen_syrk(routine == DSYR2K, lower, ta, n, k, alpha, beta, A, lda, B, ldb, C, ldc)
+            elif routine == DSYMM:
+                tasks = self.gen_symm(left, lower, m, n, alpha, beta, A, lda, B, ldb, C, ldc)
+            else:
+                tasks = self.gen_trxm(routine == DTRSM, left, lower, ta, diag.upper(), m, n, alpha, A, lda, C, ldc)
+            if tasks:
+                self.run(tasks, sync, out)
+            if sync and tasks is not None:
                 self.full_sync()
-                ta, tb = transA.upper() in "TC", transB.upper() in "TC"
-                if alpha != 0 and k > 0:
-                    self.invalidate(A, (k, m) if ta else (m, k), lda)
-                    self.invalidate(B, (n, k) if tb else (k, n), ldb)
-                self.invalidate(C, (m, n), ldc)
+                if routine == DGEMM:
+                    if alpha != 0 and k > 0:
+                        self.invalidate(A, (k, m) if ta else (m, k), lda)
+                        self.invalidate(B, (n, k) if tb else (k, n), ldb)
+                    self.invalidate(C, (m, n), ldc)
+                elif routine in (DSYRK, DSYR2K):
+                    if alpha != 0 and k > 0:
+                        self.invalidate(A, (k, n) if ta else (n, k), lda)
+                        if routine == DSYR2K:
+                            self.invalidate(B, (k, n) if ta else (n, k), ldb)
+                    self.invalidate(C, (n, n), ldc)
+                elif routine == DSYMM:
+                    if alpha != 0:
+                        ka = m if left else n
+                        self.invalidate(A, (ka, ka), lda)
+                        self.invalidate(B, (m, n), ldb)
+                    self.invalidate(C, (m, n), ldc)
+                else:
+                    ka = m if left else n
+                    if alpha != 0:
+                        self.invalidate(A, (ka, ka), lda)
+                    self.invalidate(C, (m, n), ldc)
         elif routine == COHERENT:
             self.coherent(C, m, n, ldc, out)
         elif routine == SYNC:
@@ -181,9 +210,18 @@ class Model:
             self.prefetch(C, m, n, ldc, out)
         return out
 
-    def gemm(self, ta, tb, m, n, k, alpha, beta, A, lda, B, ldb, C, ldc, sync, out):
+    # ---- task generators: program order, symbolic versions (readings in DESIGN.md)
+    def _task(self, vers, op, i, j, out, ins, skey, flops, tk):
+        """ins = [(tile, operand)] in input order; versions read now, output bumped."""
+        t = dict(gpu=self.owner(i, j), op=op, out=out, tk=tk, i=i, j=j, flops=flops, skey=skey,
+                 ins=[(tl, vers.get(id(tl), tl.ver), opnd) for (tl, opnd) in ins])
+        vers[id(out)] = vers.get(id(out), out.ver) + 1
+        t["ver"] = vers[id(out)]
+        return t
+
+    def gen_gemm(self, ta, tb, m, n, k, alpha, beta, A, lda, B, ldb, C, ldc):
         if m == 0 or n == 0 or ((alpha == 0 or k == 0) and beta == 1):
-            return
+            return None
         T = self.T
         scale = alpha == 0 or k == 0
         self.matrix(C, ldc, m, n)
@@ -192,42 +230,184 @@ class Model:
             self.matrix(B, ldb, *((n, k) if tb else (k, n)))
         tm, tn = ceil_div(m, T), ceil_div(n, T)
         tk = 0 if scale else ceil_div(k, T)
-        tasks = []  # program order (j, i, kk)
+        tmod = max(1, tm, tn)
+        vers, tasks = {}, []
         for j in range(tn):
             for i in range(tm):
                 ct = self.tile(C, ldc, i, j)
-                v0 = ct.ver
                 mt, nt = min(T, m - i * T), min(T, n - j * T)
                 if scale:
-                    ins = [(ct, v0, 2)] if beta != 0 else []
-                    tasks.append(dict(gpu=self.owner(i, j), out=ct, ver=v0 + 1, ins=ins, tk=-1, i=i,
-                                      j=j, flops=mt * nt, last=True))
+                    ins = [(ct, 2)] if beta != 0 else []
+                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
                     continue
                 for kk in range(tk):
                     kt = min(T, k - kk * T)
                     at = self.tile(A, lda, kk, i) if ta else self.tile(A, lda, i, kk)
                     bt = self.tile(B, ldb, j, kk) if tb else self.tile(B, ldb, kk, j)
-                    ins = [(at, at.ver, 0), (bt, bt.ver, 1)]
-                    if kk > 0:
-                        ins.append((ct, v0 + kk, 2))
-                    elif beta != 0:
-                        ins.append((ct, v0, 2))
-                    tasks.append(dict(gpu=self.owner(i, j), out=ct, ver=v0 + kk + 1, ins=ins, tk=kk,
-                                      i=i, j=j, flops=2 * mt * nt * kt, last=kk == tk - 1))
-        self.run(tasks, sync, out)
+                    ins = [(at, 0), (bt, 1)] + ([(ct, 2)] if (kk > 0 or beta != 0) else [])
+                    tasks.append(self._task(vers, OP_GEMM, i, j, ct, ins, (kk, (i + j + kk) % tmod, i, j, 0),
+                                            2 * mt * nt * kt, kk))
+        return tasks
+
+    def gen_syrk(self, two, lower, tr, n, k, alpha, beta, A, lda, B, ldb, C, ldc):
+        if n == 0 or ((alpha == 0 or k == 0) and beta == 1):
+            return None
+        T = self.T
+        scale = alpha == 0 or k == 0
+        self.matrix(C, ldc, n, n)
+        if not scale:
+            self.matrix(A, lda, *((k, n) if tr else (n, k)))
+            if two:
+                self.matrix(B, ldb, *((k, n) if tr else (n, k)))
+        tn = ceil_div(n, T)
+        tk = 0 if scale else ceil_div(k, T)
+        tmod = max(1, tn)
+        vers, tasks = {}, []
+
+        def opnd(X, ld, r, l):
+            return self.tile(X, ld, l, r) if tr else self.tile(X, ld, r, l)
+        for j in range(tn):
+            for i in range(tn):
+                if (i < j) if lower else (i > j):
+                    continue
+                dg = i == j
+                ct = self.tile(C, ldc, i, j)
+                mt, nt = min(T, n - i * T), min(T, n - j * T)
+                if scale:
+                    ins = [(ct, 2)] if (beta != 0 or dg) else []
+                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
+                    continue
+                first = True
+                for l in range(tk):
+                    kt = min(T, k - l * T)
+                    for s in range(2 if two else 1):
+                        xa = (B, ldb, 1) if (two and s == 1) else (A, lda, 0)
+                        xb = (B, ldb, 1) if (two and s == 0) else (A, lda, 0)
+                        at, bt = opnd(xa[0], xa[1], i, l), opnd(xb[0], xb[1], j, l)
+                        ins = [(at, xa[2]), (bt, xb[2])] + ([(ct, 2)] if (not first or beta != 0 or dg) else [])
+                        fl = kt * nt * (nt + 1) if dg else 2 * mt * nt * kt
+                        tasks.append(self._task(vers, OP_GEMM_TRI if dg else OP_GEMM, i, j, ct, ins,
+                                                (2 * l + s, (i + j + l) % tmod, i, j, 0), fl, l))
+                        first = False
+        return tasks
+
+    def gen_symm(self, left, lower, m, n, alpha, beta, A, lda, B, ldb, C, ldc):
+        if m == 0 or n == 0 or (alpha == 0 and beta == 1):
+            return None
+        T = self.T
+        scale = alpha == 0
+        ka = m if left else n
+        self.matrix(C, ldc, m, n)
+        if not scale:
+            self.matrix(A, lda, ka, ka)
+            self.matrix(B, ldb, m, n)
+        tm, tn, tl = ceil_div(m, T), ceil_div(n, T), ceil_div(ka, T)
+        tmod = max(1, tm, tn)
+        vers, tasks = {}, []
+        for j in range(tn):
+            for i in range(tm):
+                ct = self.tile(C, ldc, i, j)
+                mt, nt = min(T, m - i * T), min(T, n - j * T)
+                if scale:
+                    ins = [(ct, 2)] if beta != 0 else []
+                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
+                    continue
+                for l in range(tl):
+                    kt = min(T, ka - l * T)
+                    r, q = (i, l) if left else (l, j)
+                    in_tri = (r >= q) if lower else (r <= q)
+                    at = self.tile(A, lda, r, q) if in_tri else self.tile(A, lda, q, r)
+                    bt = self.tile(B, ldb, l, j) if left else self.tile(B, ldb, i, l)
+                    if r == q or left:
+                        ins = [(at, 0), (bt, 1)]
+                    else:
+                        ins = [(bt, 1), (at, 0)]
+                    if l > 0 or beta != 0:
+                        ins.append((ct, 2))
+                    tasks.append(self._task(vers, OP_SYMM_DIAG if r == q else OP_GEMM, i, j, ct, ins,
+                                            (l, (i + j + l) % tmod, i, j, 0), 2 * mt * nt * kt, l))
+        return tasks
+
+    def gen_trxm(self, solve, left, lower, tr, diag, m, n, alpha, A, lda, C, ldc):
+        if m == 0 or n == 0:
+            return None
+        T = self.T
+        ka = m if left else n
+        elow = lower != tr
+        self.matrix(C, ldc, m, n)
+        tm, tn, tk = ceil_div(m, T), ceil_div(n, T), ceil_div(ka, T)
+        tmod = max(1, tm, tn)
+        vers, tasks = {}, []
+        if alpha == 0:
+            for j in range(tn):
+                for i in range(tm):
+                    ct = self.tile(C, ldc, i, j)
+                    mt, nt = min(T, m - i * T), min(T, n - j * T)
+                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, [], (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
+            return tasks
+        self.matrix(A, lda, ka, ka)
+
+        def opA(r, q):
+            return self.tile(A, lda, q, r) if tr else self.tile(A, lda, r, q)
+        fwd = (left == elow) if solve else (left != elow)
+        other = tn if left else tm
+        for s in range(tk):
+            kx = s if fwd else tk - 1 - s
+            for o in range(other):
+                bi, bj = (kx, o) if left else (o, kx)
+                ot = self.tile(C, ldc, bi, bj)
+                mt, nt = min(T, m - bi * T), min(T, n - bj * T)
+                fl = mt * mt * nt if left else mt * nt * nt
+                tasks.append(self._task(vers, OP_TRSM_DIAG if solve else OP_TRMM_DIAG, bi, bj, ot,
+                                        [(opA(kx, kx), 0), (ot, 2)], (s, 0, (bi + bj + s) % tmod, bi, bj), fl, s))
+                if not solve:
+                    ph = 1
+                    for q in range(tk):
+                        contrib = (q < kx if elow else q > kx) if left else (q > kx if elow else q < kx)
+                        if not contrib:
+                            continue
+                        kt = min(T, ka - q * T)
+                        if left:
+                            ins = [(opA(kx, q), 0), (self.tile(C, ldc, q, bj), 2), (ot, 2)]
+                        else:
+                            ins = [(self.tile(C, ldc, bi, q), 2), (opA(q, kx), 0), (ot, 2)]
+                        tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins,
+                                                (s, ph, (bi + bj + s) % tmod, bi, bj), 2 * mt * nt * kt, s))
+                        ph += 1
+            if not solve:
+                continue
+            for r in range(tk):
+                if not (r > kx if fwd else r < kx):
+                    continue
+                for o in range(other):
+                    bi, bj = (r, o) if left else (o, r)
+                    ot = self.tile(C, ldc, bi, bj)
+                    mt, nt = min(T, m - bi * T), min(T, n - bj * T)
+                    kt = min(T, ka - kx * T)
+                    if left:
+                        ins = [(opA(r, kx), 0), (self.tile(C, ldc, kx, bj), 2), (ot, 2)]
+                    else:
+                        ins = [(self.tile(C, ldc, bi, kx), 2), (opA(kx, r), 0), (ot, 2)]
+                    tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins, (s, 1, (bi + bj + s) % tmod, bi, bj),
+                                            2 * mt * nt * kt, s))
+        return tasks
 
     def run(self, tasks, sync, out):
         pending = {}
+        last = {}
         for t in tasks:
             for (tl, v, _) in t["ins"]:
                 pending[(id(tl), v)] = pending.get((id(tl), v), 0) + 1
-        tmax = max([max(t["i"], t["j"]) + 1 for t in tasks] + [1])
+            o = id(t["out"])
+            if o not in last or last[o]["ver"] < t["ver"]:
+                last[o] = t
+        for t in last.values():
+            t["last"] = True
         lists = [[] for _ in range(self.G)]
         for t in tasks:
             lists[t["gpu"]].append(t)
         for d in range(self.G):
-            lists[d].sort(key=lambda t: (max(t["tk"], 0), (t["i"] + t["j"] + max(t["tk"], 0)) % tmax,
-                                         t["i"], t["j"]))
+            lists[d].sort(key=lambda t: t["skey"])
         pos = [0] * self.G
 
         def ready(t):
@@ -255,13 +435,14 @@ class Model:
             t = lists[d][pos[d]]
             deps = [-1, -1, -1, -1]
             ready_at = 0
-            for (tl, v, operand) in t["ins"]:
+            for p, (tl, v, operand) in enumerate(t["ins"]):
                 c = tl.gpus.get(d)
                 if c is None or c.ver != v:
                     self.copy_in(tl, v, d, treq, operand, out)
                 c = tl.gpus[d]
                 ready_at = max(ready_at, c.t_done)
-                deps[operand] = c.producer
+                if p < 4:
+                    deps[p] = c.producer
                 pending[(id(tl), v)] -= 1
             start = max(self.gfree[d], ready_at)
             end = start + self.nsec(t["flops"], self.rate)
@@ -269,12 +450,12 @@ class Model:
             self.hist[d].append(end)
             o = t["out"]
             out.append((self.seq, TASK, 2, o.bi, o.bj, t["tk"], t["ver"], d, d, S_NONE, 0, start, end,
-                        t["flops"], tuple(deps)))
+                        t["flops"], tuple(deps), t["op"]))
             o.ver = t["ver"]
             o.gpus = {d: Copy(t["ver"], end, self.seq, 0)}
             task_seq = self.seq
             self.seq += 1
-            if sync and t["last"]:
+            if sync and t.get("last"):
                 self.copy_out(o, d, (0, 0, o.rows, o.cols), end, task_seq, out)
             pos[d] += 1
             left -= 1

@@ -270,3 +270,87 @@ def test_dependencies_point_backwards():
     tasks = [r for r in recs if r[1] == pm.TASK]
     assert len(tasks) == 10 * 9 * 11
     assert all(r[14][0] >= 0 and r[14][1] >= 0 for r in tasks)
+
+
+# ------------------------------------------------------------------ BLAS-3 beyond GEMM (§8(f))
+def blas3_calls(routine, N, T, sync=True, alpha=1.5, beta=-0.75):
+    base = dict(routine=routine, m=N, n=N, k=N, alpha=alpha, beta=beta, A=A_ADDR, lda=N + 2, B=B_ADDR,
+                ldb=N + 1, C=C_ADDR, ldc=N, sync=sync)
+    out = []
+    if routine in (pm.DSYRK, pm.DSYR2K):
+        for uplo, tr in itertools.product("LU", "NT"):
+            out.append(dict(base, uplo=uplo, transA=tr))
+    elif routine == pm.DSYMM:
+        for side, uplo in itertools.product("LR", "LU"):
+            out.append(dict(base, side=side, uplo=uplo))
+    else:
+        for side, uplo, tr, dg in itertools.product("LR", "LU", "NT", "NU"):
+            out.append(dict(base, side=side, uplo=uplo, transA=tr, diag=dg))
+    return out
+
+
+@pytest.mark.parametrize("routine", [pm.DSYRK, pm.DSYR2K, pm.DSYMM, pm.DTRMM, pm.DTRSM])
+@pytest.mark.parametrize("G", [1, 2, 4, 8])
+def test_bit_exact_blas3(routine, G):
+    for topo_name, mode, opt in [("fig2", "ranked", True), ("uniform", "ranked", False),
+                                 ("random", "unranked", True), ("random", "home", False)]:
+        bw = TOPOS[topo_name](G)
+        flags = dict(topo=mode, optimistic=opt, window=2, tile=4)
+        for N in (13, 16):
+            for c in blas3_calls(routine, N, 4):
+                got, exp = both(bw, flags, [c])
+                assert got == exp, (routine, G, topo_name, mode, opt, N, c)
+    # alpha == 0 / beta special values / async + coherence
+    bw = TOPOS["fig2"](G)
+    flags = dict(topo="ranked", optimistic=True, window=2, tile=4)
+    for alpha, beta in [(0.0, 2.0), (0.0, 0.0), (1.5, 0.0), (1.5, 1.0)]:
+        cs = blas3_calls(routine, 11, 4, alpha=alpha, beta=beta)[:2]
+        got, exp = both(bw, flags, cs)
+        assert got == exp, (routine, G, alpha, beta)
+    cs = [dict(c, sync=False) for c in blas3_calls(routine, 12, 4)[:1]]
+    cs.append(dict(routine=pm.COHERENT, m=12, n=12, C=C_ADDR, ldc=12))
+    got, exp = both(bw, flags, cs)
+    assert got == exp
+
+
+def test_trsm_then_gemm_composition():
+    """Paper Figs. 8/9: X = L^-1 B (async), then C = X * D with no
+    intermediate coherence -- the GEMM reads X from the GPUs (no H2D of X)."""
+    G, T, N = 8, 4, 32
+    bw = TOPOS["uniform"](G)
+    flags = dict(topo="ranked", optimistic=True, window=2, tile=T)
+    calls = [dict(routine=pm.DTRSM, side="L", uplo="L", transA="N", diag="N", m=N, n=N, alpha=1.5,
+                  A=A_ADDR, lda=N, C=B_ADDR, ldc=N, sync=False),
+             dict(routine=pm.DGEMM, m=N, n=N, k=N, alpha=1.0, beta=0.0, A=B_ADDR, lda=N, B=D_ADDR, ldb=N,
+                  C=E_ADDR, ldc=N, sync=False),
+             dict(routine=pm.COHERENT, m=N, n=N, C=E_ADDR, ldc=N)]
+    got, exp = both(bw, flags, calls)
+    assert got == exp
+    gemm_recs = got[1]
+    assert not any(r[1] == pm.H2D and r[2] == 0 for r in gemm_recs)  # X never re-read from host
+    assert any(r[1] == pm.P2P and r[2] == 0 for r in gemm_recs)
+
+
+def test_triangular_task_structure():
+    """Task counts of the tiled algorithms (PLASMA structure): SYRK touches only
+    the t(t+1)/2 triangle tiles; TRSM has t diagonal solves per column of tiles and
+    t(t-1)/2 GEMM updates per column; diagonal tiles carry the diagonal ops."""
+    T, t = 4, 5
+    N = T * t
+    bw = uniform(4)
+    syrk = xk.plan_dump(xk.make_call(routine=pm.DSYRK, uplo="L", transA="N", n=N, k=N, alpha=1.0, beta=0.5,
+                                     A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True), bw, tile=T)
+    tasks = [r for r in syrk if r[1] == pm.TASK]
+    assert len(tasks) == t * (t + 1) // 2 * t
+    assert all((r[15] == pm.OP_GEMM_TRI) == (r[3] == r[4]) for r in tasks)
+    assert all(r[3] >= r[4] for r in tasks)  # lower triangle only
+    d2h = [r for r in syrk if r[1] == pm.D2H]
+    assert len(d2h) == t * (t + 1) // 2
+    trsm = xk.plan_dump(xk.make_call(routine=pm.DTRSM, side="L", uplo="L", transA="N", diag="N", m=N, n=N,
+                                     alpha=1.0, A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True), bw, tile=T)
+    tasks = [r for r in trsm if r[1] == pm.TASK]
+    assert sum(1 for r in tasks if r[15] == pm.OP_TRSM_DIAG) == t * t
+    assert sum(1 for r in tasks if r[15] == pm.OP_GEMM) == t * t * (t - 1) // 2
+    # L tiles read: only the lower triangle of A is ever copied
+    a_tiles = {(r[3], r[4]) for r in trsm if r[1] in (pm.H2D, pm.P2P) and r[2] == 0}
+    assert all(i >= j for (i, j) in a_tiles) and len(a_tiles) == t * (t + 1) // 2
