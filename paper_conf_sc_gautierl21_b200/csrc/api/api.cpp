@@ -62,6 +62,9 @@ int gemm_impl(char transA, char transB, int64_t m, int64_t n, int64_t k, double 
     c.routine = XK_ROUTINE_DGEMM;
     c.transA = is_trans(transA) ? 'T' : 'N';
     c.transB = is_trans(transB) ? 'T' : 'N';
+    c.uplo = 'L';
+    c.side = 'L';
+    c.diag = 'N';
     c.m = m;
     c.n = n;
     c.k = k;
@@ -93,10 +96,6 @@ int view_call(int routine, int64_t m, int64_t n, const double *A, int64_t lda, b
     return rt->run(c, wait);
 }
 
-int not_yet(const char *name) {
-    xk::set_error(std::string(name) + ": routine not implemented in this build (SURVEY.md §8(f) NEXT)");
-    return XK_ERR_UNSUPPORTED;
-}
 
 }  // namespace
 
@@ -161,7 +160,7 @@ int xk_dgemm_async(char transA, char transB, int64_t m, int64_t n, int64_t k, do
     return gemm_impl(transA, transB, m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, false);
 }
 
-// ---- other BLAS-3: argument checking now, tile algorithms per SURVEY.md §8(f)
+// ---- other BLAS-3: tile algorithms of PLASMA structure
 static int syrk_check(char uplo, char trans, int64_t n, int64_t k, int64_t lda, int64_t ldc) {
     if (!ok_uplo(uplo)) return -1;
     if (!ok_trans(trans)) return -2;
@@ -170,18 +169,6 @@ static int syrk_check(char uplo, char trans, int64_t n, int64_t k, int64_t lda, 
     if (lda < imax(1, is_trans(trans) ? k : n)) return -7;
     if (ldc < imax(1, n)) return -10;
     return 0;
-}
-int xk_dsyrk(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
-             int64_t lda, double beta, double *C, int64_t ldc) {
-    (void)alpha; (void)A; (void)beta; (void)C;
-    int info = syrk_check(uplo, trans, n, k, lda, ldc);
-    return info ? info : not_yet("xk_dsyrk");
-}
-int xk_dsyrk_async(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
-                   int64_t lda, double beta, double *C, int64_t ldc) {
-    (void)alpha; (void)A; (void)beta; (void)C;
-    int info = syrk_check(uplo, trans, n, k, lda, ldc);
-    return info ? info : not_yet("xk_dsyrk_async");
 }
 static int syr2k_check(char uplo, char trans, int64_t n, int64_t k, int64_t lda, int64_t ldb,
                        int64_t ldc) {
@@ -195,18 +182,6 @@ static int syr2k_check(char uplo, char trans, int64_t n, int64_t k, int64_t lda,
     if (ldc < imax(1, n)) return -12;
     return 0;
 }
-int xk_dsyr2k(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
-              int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
-    (void)alpha; (void)A; (void)B; (void)beta; (void)C;
-    int info = syr2k_check(uplo, trans, n, k, lda, ldb, ldc);
-    return info ? info : not_yet("xk_dsyr2k");
-}
-int xk_dsyr2k_async(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
-                    int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
-    (void)alpha; (void)A; (void)B; (void)beta; (void)C;
-    int info = syr2k_check(uplo, trans, n, k, lda, ldb, ldc);
-    return info ? info : not_yet("xk_dsyr2k_async");
-}
 static int symm_check(char side, char uplo, int64_t m, int64_t n, int64_t lda, int64_t ldb,
                       int64_t ldc) {
     if (!ok_side(side)) return -1;
@@ -217,18 +192,6 @@ static int symm_check(char side, char uplo, int64_t m, int64_t n, int64_t lda, i
     if (ldb < imax(1, m)) return -9;
     if (ldc < imax(1, m)) return -12;
     return 0;
-}
-int xk_dsymm(char side, char uplo, int64_t m, int64_t n, double alpha, const double *A,
-             int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
-    (void)alpha; (void)A; (void)B; (void)beta; (void)C;
-    int info = symm_check(side, uplo, m, n, lda, ldb, ldc);
-    return info ? info : not_yet("xk_dsymm");
-}
-int xk_dsymm_async(char side, char uplo, int64_t m, int64_t n, double alpha, const double *A,
-                   int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
-    (void)alpha; (void)A; (void)B; (void)beta; (void)C;
-    int info = symm_check(side, uplo, m, n, lda, ldb, ldc);
-    return info ? info : not_yet("xk_dsymm_async");
 }
 static int tr_check(char side, char uplo, char ta, char diag, int64_t m, int64_t n, int64_t lda,
                     int64_t ldb) {
@@ -242,29 +205,130 @@ static int tr_check(char side, char uplo, char ta, char diag, int64_t m, int64_t
     if (ldb < imax(1, m)) return -11;
     return 0;
 }
+
+static int run_call(xk_call_t &c, bool sync) {
+    xk::Runtime *rt = runtime();
+    if (!rt) return need_init();
+    c.sync = sync ? 1 : 0;
+    return rt->run(c, sync);
+}
+
+static int syrk_impl(bool two, char uplo, char trans, int64_t n, int64_t k, double alpha,
+                     const double *A, int64_t lda, const double *B, int64_t ldb, double beta,
+                     double *C, int64_t ldc, bool sync) {
+    int info = two ? syr2k_check(uplo, trans, n, k, lda, ldb, ldc) : syrk_check(uplo, trans, n, k, lda, ldc);
+    if (info) return info;
+    if (n == 0 || ((alpha == 0.0 || k == 0) && beta == 1.0)) return XK_OK;
+    xk_call_t c{};
+    c.routine = two ? XK_ROUTINE_DSYR2K : XK_ROUTINE_DSYRK;
+    c.uplo = up(uplo);
+    c.transA = is_trans(trans) ? 'T' : 'N';
+    c.transB = 'N';
+    c.side = 'L';
+    c.diag = 'N';
+    c.m = n;
+    c.n = n;
+    c.k = k;
+    c.alpha = alpha;
+    c.beta = beta;
+    c.A = (uint64_t)(uintptr_t)A;
+    c.lda = (uint64_t)lda;
+    c.B = (uint64_t)(uintptr_t)B;
+    c.ldb = (uint64_t)(two ? ldb : 1);
+    c.C = (uint64_t)(uintptr_t)C;
+    c.ldc = (uint64_t)ldc;
+    return run_call(c, sync);
+}
+
+static int symm_impl(char side, char uplo, int64_t m, int64_t n, double alpha, const double *A,
+                     int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc,
+                     bool sync) {
+    int info = symm_check(side, uplo, m, n, lda, ldb, ldc);
+    if (info) return info;
+    if (m == 0 || n == 0 || (alpha == 0.0 && beta == 1.0)) return XK_OK;
+    xk_call_t c{};
+    c.routine = XK_ROUTINE_DSYMM;
+    c.side = up(side);
+    c.uplo = up(uplo);
+    c.transA = c.transB = 'N';
+    c.diag = 'N';
+    c.m = m;
+    c.n = n;
+    c.k = up(side) == 'L' ? m : n;
+    c.alpha = alpha;
+    c.beta = beta;
+    c.A = (uint64_t)(uintptr_t)A;
+    c.lda = (uint64_t)lda;
+    c.B = (uint64_t)(uintptr_t)B;
+    c.ldb = (uint64_t)ldb;
+    c.C = (uint64_t)(uintptr_t)C;
+    c.ldc = (uint64_t)ldc;
+    return run_call(c, sync);
+}
+
+static int trxm_impl(bool solve, char side, char uplo, char transA, char diag, int64_t m, int64_t n,
+                     double alpha, const double *A, int64_t lda, double *B, int64_t ldb, bool sync) {
+    int info = tr_check(side, uplo, transA, diag, m, n, lda, ldb);
+    if (info) return info;
+    if (m == 0 || n == 0) return XK_OK;
+    xk_call_t c{};
+    c.routine = solve ? XK_ROUTINE_DTRSM : XK_ROUTINE_DTRMM;
+    c.side = up(side);
+    c.uplo = up(uplo);
+    c.transA = is_trans(transA) ? 'T' : 'N';
+    c.transB = 'N';
+    c.diag = up(diag);
+    c.m = m;
+    c.n = n;
+    c.k = up(side) == 'L' ? m : n;
+    c.alpha = alpha;
+    c.beta = 0.0;
+    c.A = (uint64_t)(uintptr_t)A;
+    c.lda = (uint64_t)lda;
+    c.C = (uint64_t)(uintptr_t)B;  // the output matrix of TRMM/TRSM travels as C (xk.h)
+    c.ldc = (uint64_t)ldb;
+    return run_call(c, sync);
+}
+
+int xk_dsyrk(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
+             int64_t lda, double beta, double *C, int64_t ldc) {
+    return syrk_impl(false, uplo, trans, n, k, alpha, A, lda, nullptr, 1, beta, C, ldc, true);
+}
+int xk_dsyrk_async(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
+                   int64_t lda, double beta, double *C, int64_t ldc) {
+    return syrk_impl(false, uplo, trans, n, k, alpha, A, lda, nullptr, 1, beta, C, ldc, false);
+}
+int xk_dsyr2k(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
+              int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
+    return syrk_impl(true, uplo, trans, n, k, alpha, A, lda, B, ldb, beta, C, ldc, true);
+}
+int xk_dsyr2k_async(char uplo, char trans, int64_t n, int64_t k, double alpha, const double *A,
+                    int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
+    return syrk_impl(true, uplo, trans, n, k, alpha, A, lda, B, ldb, beta, C, ldc, false);
+}
+int xk_dsymm(char side, char uplo, int64_t m, int64_t n, double alpha, const double *A,
+             int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
+    return symm_impl(side, uplo, m, n, alpha, A, lda, B, ldb, beta, C, ldc, true);
+}
+int xk_dsymm_async(char side, char uplo, int64_t m, int64_t n, double alpha, const double *A,
+                   int64_t lda, const double *B, int64_t ldb, double beta, double *C, int64_t ldc) {
+    return symm_impl(side, uplo, m, n, alpha, A, lda, B, ldb, beta, C, ldc, false);
+}
 int xk_dtrmm(char side, char uplo, char transA, char diag, int64_t m, int64_t n, double alpha,
              const double *A, int64_t lda, double *B, int64_t ldb) {
-    (void)alpha; (void)A; (void)B;
-    int info = tr_check(side, uplo, transA, diag, m, n, lda, ldb);
-    return info ? info : not_yet("xk_dtrmm");
+    return trxm_impl(false, side, uplo, transA, diag, m, n, alpha, A, lda, B, ldb, true);
 }
 int xk_dtrmm_async(char side, char uplo, char transA, char diag, int64_t m, int64_t n, double alpha,
                    const double *A, int64_t lda, double *B, int64_t ldb) {
-    (void)alpha; (void)A; (void)B;
-    int info = tr_check(side, uplo, transA, diag, m, n, lda, ldb);
-    return info ? info : not_yet("xk_dtrmm_async");
+    return trxm_impl(false, side, uplo, transA, diag, m, n, alpha, A, lda, B, ldb, false);
 }
 int xk_dtrsm(char side, char uplo, char transA, char diag, int64_t m, int64_t n, double alpha,
              const double *A, int64_t lda, double *B, int64_t ldb) {
-    (void)alpha; (void)A; (void)B;
-    int info = tr_check(side, uplo, transA, diag, m, n, lda, ldb);
-    return info ? info : not_yet("xk_dtrsm");
+    return trxm_impl(true, side, uplo, transA, diag, m, n, alpha, A, lda, B, ldb, true);
 }
 int xk_dtrsm_async(char side, char uplo, char transA, char diag, int64_t m, int64_t n, double alpha,
                    const double *A, int64_t lda, double *B, int64_t ldb) {
-    (void)alpha; (void)A; (void)B;
-    int info = tr_check(side, uplo, transA, diag, m, n, lda, ldb);
-    return info ? info : not_yet("xk_dtrsm_async");
+    return trxm_impl(true, side, uplo, transA, diag, m, n, alpha, A, lda, B, ldb, false);
 }
 
 // ---- coherence / sync

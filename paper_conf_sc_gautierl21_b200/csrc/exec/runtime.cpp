@@ -393,7 +393,8 @@ int Runtime::issue(const Rec &R) {
         Buffer *O = buf(R.key, g, true, &rc);
         if (!O) return rc;
         const int64_t idO = (int64_t)R.key * XK_MAX_GPUS + g;
-        if (R.keyA < 0) {  // scale-only task (alpha == 0 or k == 0): not batched
+        if (R.op != XK_OP_GEMM && R.op != XK_OP_GEMM_TRI) {
+            // scale / diagonal-tile ops are launched directly, after this GPU's pending batch
             if ((rc = flush_batch(g))) return rc;
             cudaStream_t s = devs_[g].ks[0];
             for (int q = 0; q < 4; ++q)
@@ -401,13 +402,44 @@ int Runtime::issue(const Rec &R) {
             for (auto &rd : O->readers)
                 if ((rc = wait_on(s, rd))) return rc;
             if ((rc = wait_on(s, O->writer))) return rc;
-            cudaError_t ke = launch_scale_tile(R.m, R.n, R.beta, O->p, O->ld, s);
-            if (ke != cudaSuccess) return cuda_fail(ke, "scale kernel launch");
+            Buffer *A = nullptr, *B = nullptr;
+            if (R.keyA >= 0 && !(A = buf(R.keyA, g, false, &rc))) return rc;
+            if (R.keyB >= 0 && !(B = buf(R.keyB, g, false, &rc))) return rc;
+            O = buf(R.key, g, false, &rc);
+            cudaError_t ke = cudaSuccess;
+            if (R.op == XK_OP_SCALE) {
+                ke = launch_scale_tri(R.m, R.n, R.beta, O->p, O->ld, R.tri, s);
+            } else if (R.op == XK_OP_TRSM_DIAG || R.op == XK_OP_TRMM_DIAG) {
+                ke = launch_trxm_tile(R.op == XK_OP_TRSM_DIAG, R.side, R.uplo, R.ta, R.diag, R.m, R.n,
+                                      R.alpha, A->p, A->ld, O->p, O->ld, s);
+            } else if (R.op == XK_OP_SYMM_DIAG) {
+                // expand the diagonal tile of A symmetrically into a scratch tile, then GEMM
+                const int64_t ka = (R.side == 'L') ? R.m : R.n;
+                const int64_t lds = (ka + 15) / 16 * 16;
+                double *S = alloc(g, (size_t)lds * ka * 8, &rc);
+                if (!S) return rc;
+                scratch_.push_back({g, {S, (size_t)lds * ka * 8}});
+                ke = launch_symm_expand(ka, A->p, A->ld, R.uplo, S, lds, s);
+                if (ke == cudaSuccess) {
+                    if (R.side == 'L')
+                        ke = launch_dgemm_tile(false, false, R.m, R.n, R.k, R.alpha, S, lds, B->p, B->ld, R.beta,
+                                               O->p, O->ld, s);
+                    else
+                        ke = launch_dgemm_tile(false, false, R.m, R.n, R.k, R.alpha, B->p, B->ld, S, lds, R.beta,
+                                               O->p, O->ld, s);
+                }
+            } else {
+                set_error("internal: unknown tile op");
+                return XK_ERR_INTERNAL;
+            }
+            if (ke != cudaSuccess) return cuda_fail(ke, "tile kernel launch");
             Ev ev;
             if ((rc = record(s, g, &ev))) return rc;
             seq_ev_[r.seq] = ev;
             O->writer = ev;
             O->readers.clear();
+            if (A) add_reader(*A, ev);
+            if (B) add_reader(*B, ev);
             stats.tasks[g]++;
             stats.flops[g] += r.work;
             stats.kernel_launches++;
@@ -480,7 +512,7 @@ int Runtime::flush_batch(int g) {
         for (auto &rd : O->readers)
             if ((rc = wait_on(s, rd))) return rc;
         if ((rc = wait_on(s, O->writer))) return rc;
-        tb.t[q] = TileTask{A->p, B->p, O->p, A->ld, B->ld, O->ld, R.m, R.n, R.k, R.alpha, R.beta};
+        tb.t[q] = TileTask{A->p, B->p, O->p, A->ld, B->ld, O->ld, R.m, R.n, R.k, R.alpha, R.beta, R.tri};
         flops += R.r.work;
     }
     cudaEvent_t t0 = nullptr, t1 = nullptr;
@@ -722,6 +754,8 @@ int Runtime::sync_all() {
         for (cudaEvent_t e : ev_used_[g]) ev_pool_[g].push_back(e);
         ev_used_[g].clear();
     }
+    for (auto &sc : scratch_) free_buf(sc.first, sc.second.first, sc.second.second);
+    scratch_.clear();
     release_internal_pins();
     return XK_OK;
 }
@@ -732,14 +766,43 @@ int Runtime::run(const xk_call_t &call, bool wait) {
     int rc;
     // page-lock the operands the call touches (excluded from timings when the caller
     // registered them first with xk_register)
-    if (call.routine == XK_ROUTINE_DGEMM) {
-        bool ta = call.transA == 'T' || call.transA == 'C', tb = call.transB == 'T' || call.transB == 'C';
-        if (call.alpha != 0.0 && call.k > 0) {
-            if ((rc = ensure_pinned(call.A, ta ? call.k : call.m, ta ? call.m : call.k, (int64_t)call.lda))) return rc;
-            if ((rc = ensure_pinned(call.B, tb ? call.n : call.k, tb ? call.k : call.n, (int64_t)call.ldb))) return rc;
+    {
+        const bool ta = call.transA == 'T' || call.transA == 'C', tb = call.transB == 'T' || call.transB == 'C';
+        const bool left = call.side == 'L';
+        const int64_t m = call.m, n = call.n, k = call.k;
+        auto pin = [&](uint64_t p, int64_t r, int64_t c, uint64_t ld) { return ensure_pinned(p, r, c, (int64_t)ld); };
+        switch (call.routine) {
+        case XK_ROUTINE_DGEMM:
+            if (call.alpha != 0.0 && k > 0) {
+                if ((rc = pin(call.A, ta ? k : m, ta ? m : k, call.lda))) return rc;
+                if ((rc = pin(call.B, tb ? n : k, tb ? k : n, call.ldb))) return rc;
+            }
+            break;
+        case XK_ROUTINE_DSYRK:
+        case XK_ROUTINE_DSYR2K:
+            if (call.alpha != 0.0 && k > 0) {
+                if ((rc = pin(call.A, ta ? k : n, ta ? n : k, call.lda))) return rc;
+                if (call.routine == XK_ROUTINE_DSYR2K && (rc = pin(call.B, ta ? k : n, ta ? n : k, call.ldb))) return rc;
+            }
+            break;
+        case XK_ROUTINE_DSYMM:
+            if (call.alpha != 0.0) {
+                if ((rc = pin(call.A, left ? m : n, left ? m : n, call.lda))) return rc;
+                if ((rc = pin(call.B, m, n, call.ldb))) return rc;
+            }
+            break;
+        case XK_ROUTINE_DTRMM:
+        case XK_ROUTINE_DTRSM:
+            if (call.alpha != 0.0 && (rc = pin(call.A, left ? m : n, left ? m : n, call.lda))) return rc;
+            break;
+        default:
+            break;
         }
     }
-    if ((rc = ensure_pinned(call.C, call.m, call.n, (int64_t)call.ldc))) return rc;
+    {
+        const bool sy = call.routine == XK_ROUTINE_DSYRK || call.routine == XK_ROUTINE_DSYR2K;
+        if ((rc = ensure_pinned(call.C, sy ? call.n : call.m, call.n, (int64_t)call.ldc))) return rc;
+    }
     std::vector<Rec> recs;
     std::string err;
     rc = planner_->plan(call, recs, err);
@@ -752,7 +815,7 @@ int Runtime::run(const xk_call_t &call, bool wait) {
         if ((rc = issue(r))) return rc;
     for (size_t g = 0; g < batch_.size(); ++g)
         if ((rc = flush_batch((int)g))) return rc;
-    if (call.routine == XK_ROUTINE_DGEMM && call.sync) {
+    if (call.routine <= XK_ROUTINE_DTRSM && call.sync) {
         // the planner already passed its full sync point and invalidated the operands
         if ((rc = sync_all())) return rc;
         release_invalid();

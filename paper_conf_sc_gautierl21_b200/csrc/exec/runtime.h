@@ -119,6 +119,7 @@ private:
     std::vector<Ev> pending_d2h_;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ktimers_;
     std::vector<int64_t> ktimer_flops_;
+    std::vector<std::pair<int, std::pair<double *, size_t>>> scratch_;  // freed at the next full sync
     std::map<uintptr_t, size_t> registered_;    // user-registered host ranges
     std::map<uintptr_t, size_t> internal_reg_;  // registered by the library on first use
     int cur_dev_ = -1;

@@ -137,6 +137,9 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
     const int tiles_m = (int)((t.M + BM - 1) / BM);
     const int64_t m0 = (int64_t)(local % tiles_m) * BM, n0 = (int64_t)(local / tiles_m) * BN;
     const int64_t M = t.M, N = t.N, K = t.K;
+    const int tri = t.tri;
+    // diagonal tiles of SYRK/SYR2K: CTAs entirely outside the written triangle do nothing
+    if ((tri == 1 && m0 + BM - 1 < n0) || (tri == 2 && n0 + BN - 1 < m0)) return;
 
     extern __shared__ __align__(128) double smem[];
     const uint32_t sA0 = smem_u32(smem);
@@ -238,6 +241,7 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
             for (int h = 0; h < 2; ++h) {
                 const int64_t c = n0 + wn + j * 8 + fc * 2 + h;
                 if (c >= N) continue;
+                if ((tri == 1 && r < c) || (tri == 2 && r > c)) continue;
                 double *p = C + r + c * ldc;
                 double v = alpha * acc[i][j][h];
                 if (beta != 0.0) v = fma(beta, *p, v);
@@ -349,7 +353,7 @@ cudaError_t launch_dgemm_tile(bool ta, bool tb, int64_t M, int64_t N, int64_t K,
     if (alpha == 0.0 || K <= 0) return launch_scale_tile(M, N, beta, C, ldc, st);
     TileBatch b;
     b.n = 1;
-    b.t[0] = TileTask{A, B, C, lda, ldb, ldc, M, N, K, alpha, beta};
+    b.t[0] = TileTask{A, B, C, lda, ldb, ldc, M, N, K, alpha, beta, 0};
     return launch_dgemm_batch(ta, tb, b, st);
 }
 

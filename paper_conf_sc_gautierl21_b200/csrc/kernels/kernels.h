@@ -13,6 +13,7 @@ struct TileTask {
     int64_t lda, ldb, ldc;
     int64_t M, N, K;
     double alpha, beta;
+    int tri;  // 0 full tile; 1 / 2: write only the lower / upper triangle (SYRK diagonal tiles)
 };
 
 // A batch of independent tile tasks launched as one grid (grouped GEMM); passed by value
@@ -33,4 +34,15 @@ cudaError_t launch_dgemm_tile(bool ta, bool tb, int64_t M, int64_t N, int64_t K,
 // C = beta*C (beta == 0: C = 0, C not read).
 cudaError_t launch_scale_tile(int64_t M, int64_t N, double beta, double *C, int64_t ldc,
                               cudaStream_t st);
+// Diagonal-tile TRSM (solve) / TRMM (multiply) in place on B (trxm_tile.cu):
+//   side 'L': B = alpha*op(A)^-1*B or alpha*op(A)*B;  'R': B*op(A)^-1 / B*op(A).
+cudaError_t launch_trxm_tile(bool solve, char side, char uplo, char transA, char diag, int64_t M,
+                             int64_t N, double alpha, const double *A, int64_t lda, double *B,
+                             int64_t ldb, cudaStream_t st);
+// S = sym(A) (n x n) from the uplo triangle of A.
+cudaError_t launch_symm_expand(int64_t n, const double *A, int64_t lda, char uplo, double *S,
+                               int64_t lds, cudaStream_t st);
+// C = beta*C on the tri triangle only (tri 0: whole tile).
+cudaError_t launch_scale_tri(int64_t M, int64_t N, double beta, double *C, int64_t ldc, int tri,
+                             cudaStream_t st);
 }  // namespace xk

@@ -1,0 +1,248 @@
+"""GPU parity of xk_dsyrk / xk_dsyr2k / xk_dsymm / xk_dtrmm / xk_dtrsm (SURVEY.md §8(f) rows
+f1, f2, f4) against the CPU oracle, through the C ABI.
+
+Tolerances (north_star / DESIGN.md Q13): elementwise 4*k*2^-53*(|alpha||A||B|+|beta||C|)
+(SYR2K: 2k), relative Frobenius <= 1e-13; TRSM additionally the componentwise residual bound
+|op(L) X - alpha B| <= 4*m*2^-53*(|op(L)||X| + |alpha||B|).  "Not referenced" rules are checked
+with NaN poisoning; the untouched triangle of C (SYRK/SYR2K) must come back bit for bit.
+Multi-GPU logic runs in logical-device mode (G logical GPUs on the one B200).
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import inputs
+import oracle
+import paper_conf_sc_gautierl21_b200 as xk
+
+pytestmark = pytest.mark.gpu
+EPS = 2.0 ** -53
+
+
+def fmat(a):
+    return np.asfortranarray(a, dtype=np.float64)
+
+
+def tri_mask(n, lower):
+    return np.tril(np.ones((n, n), bool)) if lower else np.triu(np.ones((n, n), bool))
+
+
+@pytest.fixture(params=[1, 4], ids=["G1", "G4"])
+def lib(request):
+    G = request.param
+    xk.init(ngpus=G, phys=[0] * G, tile=128, probe=False)
+    yield G
+    xk.finalize()
+
+
+@pytest.mark.parametrize("uplo,trans", list(itertools.product("LU", "NT")))
+def test_syrk_syr2k(lib, uplo, trans):
+    n, k = 300, 200
+    lower = uplo == "L"
+    shp = (n, k) if trans == "N" else (k, n)
+    A = inputs.uniform(1, *shp); B = inputs.uniform(2, *shp)
+    C0 = inputs.uniform(3, n, n)
+    msk = tri_mask(n, lower)
+    opA = A if trans == "N" else A.T
+    opB = B if trans == "N" else B.T
+    for alpha, beta in [(1.5, -0.75), (1.5, 0.0), (0.0, 0.5)]:
+        C = C0.copy(order="F")
+        if beta == 0.0:
+            C[msk] = np.nan  # triangle not read when beta == 0
+        C[~msk] = np.nan     # other triangle never read, must come back bit for bit
+        Cin = C.copy(order="F")
+        assert xk.dsyrk(uplo, trans, n, k, alpha, A, shp[0], beta, C, n) == 0
+        ref = C0.copy(order="F")
+        oracle.dsyrk(uplo, trans, n, k, alpha, A, beta, ref)
+        bound = 4 * k * EPS * (abs(alpha) * (np.abs(opA) @ np.abs(opA).T) + abs(beta) * np.abs(C0))
+        assert np.all(np.abs(C - ref)[msk] <= bound[msk]), (alpha, beta)
+        assert np.array_equal(C[~msk], Cin[~msk], equal_nan=True)
+        # SYR2K
+        C = Cin.copy(order="F")
+        assert xk.dsyr2k(uplo, trans, n, k, alpha, A, shp[0], B, shp[0], beta, C, n) == 0
+        ref = C0.copy(order="F")
+        oracle.dsyr2k(uplo, trans, n, k, alpha, A, B, beta, ref)
+        mag = np.abs(opA) @ np.abs(opB).T + np.abs(opB) @ np.abs(opA).T
+        bound = 4 * 2 * k * EPS * (abs(alpha) * mag + abs(beta) * np.abs(C0))
+        assert np.all(np.abs(C - ref)[msk] <= bound[msk]), (alpha, beta)
+        assert np.array_equal(C[~msk], Cin[~msk], equal_nan=True)
+
+
+@pytest.mark.parametrize("side,uplo", list(itertools.product("LR", "LU")))
+def test_symm(lib, side, uplo):
+    m, n = 300, 230
+    ka = m if side == "L" else n
+    A = inputs.uniform(1, ka, ka)
+    Ap = A.copy(order="F")
+    Ap[~tri_mask(ka, uplo == "L")] = np.nan  # only the uplo triangle is read
+    B = inputs.uniform(2, m, n); C0 = inputs.uniform(3, m, n)
+    C = C0.copy(order="F")
+    assert xk.dsymm(side, uplo, m, n, 1.5, Ap, ka, B, m, -0.75, C, m) == 0
+    ref = C0.copy(order="F")
+    oracle.dsymm(side, uplo, m, n, 1.5, Ap, B, -0.75, ref)
+    S = np.where(tri_mask(ka, uplo == "L"), A, A.T)
+    mag = (np.abs(S) @ np.abs(B)) if side == "L" else (np.abs(B) @ np.abs(S))
+    assert np.all(np.abs(C - ref) <= 4 * ka * EPS * (1.5 * mag + 0.75 * np.abs(C0)))
+    assert np.linalg.norm(C - ref) <= 1e-13 * np.linalg.norm(ref)
+
+
+FLAGS = list(itertools.product("LR", "LU", "NT", "NU"))
+
+
+def tri_of(L, lower, unit):
+    T = np.where(tri_mask(L.shape[0], lower), np.nan_to_num(L, nan=0.0), 0.0)
+    if unit:
+        T[np.diag_indices(L.shape[0])] = 1.0
+    return T
+
+
+@pytest.mark.parametrize("side,uplo,ta,diag", FLAGS)
+def test_trmm_trsm(lib, side, uplo, ta, diag):
+    m, n = 300, 200
+    ka = m if side == "L" else n
+    lower, unit = uplo == "L", diag == "U"
+    L = inputs.tri_dd(4, ka, lower=lower, fill=np.nan)  # Q9 factor, opposite triangle NaN
+    if unit:
+        L[np.diag_indices(ka)] = np.nan  # diag='U': the diagonal is not read
+    B0 = inputs.uniform(2, m, n)
+    T = tri_of(L, lower, unit)
+    opT = T.T if ta == "T" else T
+    # TRMM
+    X = B0.copy(order="F")
+    assert xk.dtrmm(side, uplo, ta, diag, m, n, 1.5, L, ka, X, m) == 0
+    ref = B0.copy(order="F")
+    oracle.dtrmm(side, uplo, ta, diag, m, n, 1.5, L, ref)
+    mag = (np.abs(opT) @ np.abs(B0)) if side == "L" else (np.abs(B0) @ np.abs(opT))
+    assert np.all(np.abs(X - ref) <= 4 * ka * EPS * 1.5 * mag)
+    # TRSM
+    X = B0.copy(order="F")
+    assert xk.dtrsm(side, uplo, ta, diag, m, n, 1.5, L, ka, X, m) == 0
+    ref = B0.copy(order="F")
+    oracle.dtrsm(side, uplo, ta, diag, m, n, 1.5, L, ref)
+    assert np.linalg.norm(X - ref) <= 1e-13 * np.linalg.norm(ref)
+    R = (opT @ X - 1.5 * B0) if side == "L" else (X @ opT - 1.5 * B0)
+    magr = (np.abs(opT) @ np.abs(X)) if side == "L" else (np.abs(X) @ np.abs(opT))
+    assert np.all(np.abs(R) <= 4 * ka * EPS * (magr + 1.5 * np.abs(B0)) * 1.0000001)
+
+
+def test_trsm_bidiagonal_exact(lib):
+    """L = D(I - S), D = diag(2^p): X = alpha * prefix sums of D^-1 B exactly (bitwise)."""
+    m, n = 333, 70
+    p = (np.arange(m) % 5) - 2
+    L = fmat(np.diag(2.0 ** p) @ (np.eye(m) - np.diag(np.ones(m - 1), -1)))
+    L[np.triu_indices(m, 1)] = np.nan
+    B0 = inputs.integers(7, m, n)
+    X = B0.copy(order="F")
+    assert xk.dtrsm("L", "L", "N", "N", m, n, 2.0, L, m, X, m) == 0
+    assert np.array_equal(X, 2.0 * np.cumsum((2.0 ** -p)[:, None] * B0, axis=0))
+
+
+def test_trmm_exact_integers(lib):
+    m, n = 260, 190
+    A = inputs.integers(3, m, m, lo=-2, span=5)
+    B0 = inputs.integers(4, m, n)
+    for side, uplo, ta in [("L", "L", "N"), ("L", "U", "T"), ("R", "L", "T"), ("R", "U", "N")]:
+        ka = m if side == "L" else n
+        Ak = A[:ka, :ka].copy(order="F")
+        Bs = B0[:m, :n].copy(order="F")
+        X = Bs.copy(order="F")
+        assert xk.dtrmm(side, uplo, ta, "N", m, n, -2.0, Ak, ka, X, m) == 0
+        ref = Bs.copy(order="F")
+        oracle.dtrmm(side, uplo, ta, "N", m, n, -2.0, Ak, ref)
+        assert np.array_equal(X, ref), (side, uplo, ta)
+
+
+def test_trsm_gemm_composition():
+    """Paper Figs. 8/9 composition: X = L^-1 B async, then C = X*D async without
+    intermediate coherence; only the final C is made coherent.  Same numbers as the
+    synchronous path, and no H2D of X in the second call."""
+    G, T, N = 4, 128, 384
+    L = inputs.tri_dd(4, N, lower=True, fill=np.nan)
+    B0 = inputs.uniform(2, N, N); D = inputs.uniform(5, N, N)
+    xk.init(ngpus=G, phys=[0] * G, tile=T, probe=False)
+    try:
+        Xs = B0.copy(order="F"); Cs = np.zeros((N, N), order="F")
+        xk.dtrsm("L", "L", "N", "N", N, N, 1.5, L, N, Xs, N)
+        xk.dgemm("N", "N", N, N, N, 1.0, Xs, N, D, N, 0.0, Cs, N)
+        X = B0.copy(order="F"); C = np.full((N, N), -3.0, order="F")
+        xk.reset_stats()
+        xk.dtrsm("L", "L", "N", "N", N, N, 1.5, L, N, X, N, asynchronous=True)
+        h1 = sum(xk.get_stats()["h2d_bytes"])
+        xk.dgemm_async("N", "N", N, N, N, 1.0, X, N, D, N, 0.0, C, N)
+        h2 = sum(xk.get_stats()["h2d_bytes"]) - h1
+        assert h2 == 8 * N * N  # only D crosses PCIe; X comes from the GPUs
+        xk.memory_coherent_sync(N, N, C, N)
+        assert np.array_equal(C, Cs)
+        xk.memory_coherent_sync(N, N, X, N)
+        assert np.array_equal(X, Xs)
+    finally:
+        xk.finalize()
+
+
+@pytest.mark.parametrize("routine", ["syrk", "syr2k"])
+def test_config3_n32768_sampled(routine):
+    """BASELINE configs[2] shape (N=32768, lower, NoTrans, T=2048), one GPU: sampled lower
+    entries vs the oracle's dot loop (SYRK entry = GEMM entry of A*A^T)."""
+    N, T = 32768, 2048
+    A = inputs.uniform(1, N, N); B = inputs.uniform(2, N, N) if routine == "syr2k" else None
+    C0 = inputs.uniform(3, N, N)
+    C = C0.copy(order="F")
+    xk.init(ngpus=1, tile=T, probe=False)
+    try:
+        for X in (A, B, C):
+            if X is not None:
+                xk.register(X)
+        if routine == "syrk":
+            assert xk.dsyrk("L", "N", N, N, 1.5, A, N, -0.75, C, N) == 0
+        else:
+            assert xk.dsyr2k("L", "N", N, N, 1.5, A, N, B, N, -0.75, C, N) == 0
+    finally:
+        xk.finalize()
+    rng = np.random.default_rng(3)
+    ii = rng.integers(0, N, 3000); jj = rng.integers(0, N, 3000)
+    ii, jj = np.maximum(ii, jj), np.minimum(ii, jj)
+    if routine == "syrk":
+        ref = oracle.dgemm_sampled("N", "T", N, 1.5, A, A, -0.75, C0[ii, jj], ii, jj)
+        mag = 1.5 * np.einsum("qk,qk->q", np.abs(A[ii, :]), np.abs(A[jj, :])) + 0.75 * np.abs(C0[ii, jj])
+        kk = N
+    else:
+        r1 = oracle.dgemm_sampled("N", "T", N, 1.5, A, B, -0.75, C0[ii, jj], ii, jj)
+        r2 = oracle.dgemm_sampled("N", "T", N, 1.5, B, A, 0.0, C0[ii, jj], ii, jj)
+        ref = r1 + r2
+        mag = 1.5 * (np.einsum("qk,qk->q", np.abs(A[ii, :]), np.abs(B[jj, :])) +
+                     np.einsum("qk,qk->q", np.abs(B[ii, :]), np.abs(A[jj, :]))) + 0.75 * np.abs(C0[ii, jj])
+        kk = 2 * N
+    assert np.all(np.abs(C[ii, jj] - ref) <= 4 * kk * EPS * mag * 1.0000001)
+    up = rng.integers(0, N, 2000), rng.integers(0, N, 2000)
+    ui, uj = np.minimum(*up), np.maximum(*up)
+    sel = ui < uj
+    assert np.array_equal(C[ui[sel], uj[sel]], C0[ui[sel], uj[sel]])  # upper triangle untouched
+
+
+@pytest.mark.parametrize("routine", ["trsm", "trmm"])
+def test_config4_n32768_sampled(routine):
+    """BASELINE configs[3] shape (N=32768, left, lower, NoTrans, non-unit, T=2048), one GPU:
+    TRSM residual bound on sampled columns; TRMM sampled entries vs the dot loop."""
+    N, T = 32768, 2048
+    L = inputs.tri_dd(4, N, lower=True, fill=0.0)
+    B0 = inputs.uniform(2, N, N)
+    X = B0.copy(order="F")
+    xk.init(ngpus=1, tile=T, probe=False)
+    try:
+        xk.register(L); xk.register(X)
+        f = xk.dtrsm if routine == "trsm" else xk.dtrmm
+        assert f("L", "L", "N", "N", N, N, 1.5, L, N, X, N) == 0
+    finally:
+        xk.finalize()
+    rng = np.random.default_rng(4)
+    cols = rng.integers(0, N, 6)
+    for j in cols:
+        if routine == "trsm":
+            r = L @ X[:, j] - 1.5 * B0[:, j]
+            bound = 4 * N * EPS * (np.abs(L) @ np.abs(X[:, j]) + 1.5 * np.abs(B0[:, j]))
+            assert np.all(np.abs(r) <= bound * 1.0000001)
+        else:
+            ref = 1.5 * (L @ B0[:, j])
+            bound = 4 * N * EPS * 1.5 * (np.abs(L) @ np.abs(B0[:, j]))
+            assert np.all(np.abs(X[:, j] - ref) <= bound + 4 * N * EPS * np.abs(ref))
