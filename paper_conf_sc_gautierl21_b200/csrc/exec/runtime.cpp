@@ -66,6 +66,7 @@ int Runtime::init(const xk_config_t &cfg) {
     }
     int ks = cfg.kstreams > 0 ? std::min(cfg.kstreams, kMaxKStreams) : 2;
     cfg_.kstreams = ks;
+    nks_ = std::max(ks, 4);  // streams created: batches use the first ks, diagonal ops all
     // peer access between distinct physical devices (NVLink / NVSwitch)
     for (int a = 0; a < G; ++a)
         for (int b = 0; b < G; ++b) {
@@ -85,7 +86,7 @@ int Runtime::init(const xk_config_t &cfg) {
         XK_CK(cudaStreamCreateWithFlags(&d.h2d, cudaStreamNonBlocking));
         XK_CK(cudaStreamCreateWithFlags(&d.d2h, cudaStreamNonBlocking));
         XK_CK(cudaStreamCreateWithFlags(&d.p2p, cudaStreamNonBlocking));
-        for (int k = 0; k < ks; ++k) XK_CK(cudaStreamCreateWithFlags(&d.ks[k], cudaStreamNonBlocking));
+        for (int k = 0; k < nks_; ++k) XK_CK(cudaStreamCreateWithFlags(&d.ks[k], cudaStreamNonBlocking));
     }
     cur_dev_ = -1;
     ev_pool_.assign(G, {});
@@ -396,7 +397,10 @@ int Runtime::issue(const Rec &R) {
         if (R.op != XK_OP_GEMM && R.op != XK_OP_GEMM_TRI) {
             // scale / diagonal-tile ops are launched directly, after this GPU's pending batch
             if ((rc = flush_batch(g))) return rc;
-            cudaStream_t s = devs_[g].ks[0];
+            // independent diagonal-tile ops of one step (e.g. the TRSM solves of every column
+            // of tiles) spread over all kernel streams so they overlap
+            const uint64_t h = (uint64_t)(e.bi * 7919 + e.bj * 104729);
+            cudaStream_t s = devs_[g].ks[h % (uint64_t)nks_];
             for (int q = 0; q < 4; ++q)
                 if ((rc = wait_dep(s, r.dep[q]))) return rc;
             for (auto &rd : O->readers)
@@ -727,7 +731,7 @@ int Runtime::sync_all() {
         XK_CK(cudaSetDevice(d.phys));
         XK_CK(cudaStreamSynchronize(d.h2d));
         XK_CK(cudaStreamSynchronize(d.p2p));
-        for (int k = 0; k < cfg_.kstreams; ++k) XK_CK(cudaStreamSynchronize(d.ks[k]));
+        for (int k = 0; k < nks_; ++k) XK_CK(cudaStreamSynchronize(d.ks[k]));
         XK_CK(cudaStreamSynchronize(d.d2h));
     }
     cur_dev_ = -1;
@@ -853,7 +857,7 @@ int Runtime::finalize() {
         cudaStreamDestroy(d.h2d);
         cudaStreamDestroy(d.d2h);
         cudaStreamDestroy(d.p2p);
-        for (int k = 0; k < cfg_.kstreams; ++k) cudaStreamDestroy(d.ks[k]);
+        for (int k = 0; k < nks_; ++k) cudaStreamDestroy(d.ks[k]);
         for (cudaEvent_t e : ev_pool_[g]) cudaEventDestroy(e);
     }
     bufs_.clear();

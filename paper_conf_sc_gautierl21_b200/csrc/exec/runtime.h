@@ -126,6 +126,7 @@ private:
     std::vector<PendingBatch> batch_;
     std::vector<int64_t> batch_count_;
     int max_batch_ = kMaxBatch;
+    int nks_ = 4;  // kernel streams created per GPU
 };
 
 Runtime *runtime();  // global instance (nullptr before xk_init)
