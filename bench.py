@@ -336,7 +336,7 @@ def run_xk(args, rank, ws):
     achieved = flops_per_launch / (avg_ms * 1e-3) / 1e12 if avg_ms > 0 else None
     roof = {"bound": "tensor", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
             "frac": (achieved / FP64_PEAK_TFLOPS) if achieved else None, "traffic": traffic_from_profiles(T),
-            "kernel": "dgemm_tile_kernel (FP64 DMMA.8x8x4 via mma.sync.m8n8k4.f64)",
+            "kernel": "dgemm_tma_kernel (grouped launch; TMA + mbarrier pipeline; FP64 DMMA.8x8x4 via mma.sync.m8n8k4.f64)",
             "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 x 1965 MHz (no FP64 entry in "
                            "MEASURED_PEAKS.json); DMMA microbenchmark on this pool measured 37.07",
             "per_launch": "one grouped launch = a batch of tile tasks, 2*T^3 flops each (T=%d); %.3g flops "

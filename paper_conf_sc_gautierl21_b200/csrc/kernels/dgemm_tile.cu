@@ -326,8 +326,39 @@ __global__ void scale_tile_kernel(int64_t M, int64_t N, double beta, double *C, 
 
 }  // namespace
 
+bool tma_enabled() {
+    static int on = -1;
+    if (on < 0) {
+        const char *e = getenv("XK_TMA");
+        on = (e && *e) ? atoi(e) : 1;
+    }
+    return on != 0;
+}
+
+// Grouped launch: the TMA + mbarrier kernel when every operand can be described by a
+// tensor map (16-byte aligned base and ld), else the cp.async kernel.
 cudaError_t launch_dgemm_batch(bool ta, bool tb, TileBatch &b, cudaStream_t st) {
     if (b.n <= 0) return cudaSuccess;
+    if (tma_enabled() && b.n <= kMaxTmaBatch) {
+        static thread_local TmaBatch tb_;
+        tb_.n = b.n;
+        bool ok = true;
+        for (int q = 0; q < b.n && ok; ++q) {
+            const TileTask &t = b.t[q];
+            TmaTask &u = tb_.t[q];
+            ok = make_tma_operand(&u.mapA, t.A, ta ? t.K : t.M, ta ? t.M : t.K, t.lda, !ta, tma_bm()) &&
+                 make_tma_operand(&u.mapB, t.B, tb ? t.N : t.K, tb ? t.K : t.N, t.ldb, tb, tma_bn());
+            u.C = t.C;
+            u.ldc = t.ldc;
+            u.M = t.M;
+            u.N = t.N;
+            u.K = t.K;
+            u.alpha = t.alpha;
+            u.beta = t.beta;
+            u.tri = t.tri;
+        }
+        if (ok) return launch_dgemm_tma(ta, tb, tb_, st);
+    }
     // 16-byte cp.async needs 16-byte aligned columns of both operands in every task
     bool v2 = true;
     for (int q = 0; q < b.n; ++q)

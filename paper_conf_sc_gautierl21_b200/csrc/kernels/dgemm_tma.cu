@@ -1,0 +1,299 @@
+// dgemm_tma.cu -- FP64 tile GEMM for sm_100a with TMA loads and an mbarrier pipeline.
+//
+//   D = alpha * op(A) * op(B) + beta * C on column-major device tiles (same operation and
+//   batching as dgemm_tile.cu).
+//
+// Why a second kernel: the cp.async kernel spends ~14% of its issue slots/time on per-thread
+// address math, the per-k-block __syncthreads and cp.async waits (profiles/r01_*).  Here one
+// thread streams whole operand boxes with the Tensor Memory Accelerator
+// (cp.async.bulk.tensor.2d, zero-filled out of bounds so ragged tiles need no predication),
+// each stage completes on a transaction-count mbarrier, and warps release stages through an
+// "empty" mbarrier: no CTA-wide barrier in the main loop.
+//
+// Shared-memory layout: TMA 128-byte swizzle (16-byte chunk index XOR row % 8).  mn-contiguous
+// operands are loaded as 16(mn) x 16(k) boxes (rows = k), k-contiguous operands as one
+// 16(k) x BMN box (rows = mn).  The m8n8k4 fragments read k in a permuted order
+// sigma(s, q) = X[s] ^ Q[q], X = {0,1,4,5}, Q = {0,3,12,15}: it partitions the 16 k of a
+// stage into 4 steps and makes every 8-byte fragment read conflict-free for BOTH swizzled
+// layouts.  A and B use the same permutation, so each step still sums over
+// matching k; only the (legal) summation order changes.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdlib.h>
+
+#include "kernels/kernels.h"
+
+namespace xk {
+namespace {
+
+constexpr int BK = 16;
+constexpr int BM = 64, BN = 128;   // CTA tile
+constexpr int WM = 32, WN = 32;    // warp tile
+constexpr int NWM = BM / WM, NWN = BN / WN, NWARPS = NWM * NWN;
+constexpr int NTHREADS = NWARPS * 32;
+constexpr int STAGES = 4;
+constexpr int A_BYTES = BM * BK * 8, B_BYTES = BN * BK * 8, STAGE_BYTES = A_BYTES + B_BYTES;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(bar),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map, int c0, int c1,
+                                            uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(dst),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(bar)
+        : "memory");
+}
+__device__ __forceinline__ void dmma(double (&c)[2], double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c[0]), "+d"(c[1])
+                 : "d"(a), "d"(b));
+}
+
+// Byte offset of fragment element (mn = base8 + fr, k = x ^ qk) inside an operand region of
+// one stage, split as lane_part ^ const_part: the two parts occupy disjoint bit ranges except
+// where the swizzle XORs them, so each fragment address is one XOR with a compile-time
+// constant (base8 = warp offset + 8*i is a multiple of 8; x in {0,1,4,5}; qk in {0,3,12,15}).
+//   mn-contiguous (16 x 16 boxes, rows = k): off = (mn>>4)*2048 + k*128 + ((((mn&15)>>1) ^ (k&7))<<4) + (mn&1)*8
+//   k-contiguous  (rows = mn)            : off = mn*128 + (((k>>1) ^ (mn&7))<<4) + (k&1)*8
+template <bool MN_CONTIG>
+__device__ __forceinline__ uint32_t lane_part(int fr, int qk) {
+    if (MN_CONTIG) return (uint32_t)((qk << 7) | ((((fr >> 1) ^ (qk & 7)) & 7) << 4) | ((fr & 1) << 3));
+    return (uint32_t)((fr << 7) | ((((qk >> 1) ^ fr) & 7) << 4) | ((qk & 1) << 3));
+}
+template <bool MN_CONTIG>
+__device__ __forceinline__ uint32_t const_part(int base8, int x) {
+    if (MN_CONTIG) return (uint32_t)(((base8 >> 4) << 11) | (x << 7) | (((((base8 & 8) >> 1) ^ x) & 7) << 4));
+    return (uint32_t)((base8 << 7) | (((x >> 1) & 7) << 4) | ((x & 1) << 3));
+}
+
+template <bool MN_CONTIG, int BMN>
+__device__ __forceinline__ void issue_operand(uint32_t dst, const CUtensorMap *map, int mn0, int k0,
+                                              uint32_t bar) {
+    if (MN_CONTIG) {
+#pragma unroll
+        for (int q = 0; q < BMN / 16; ++q) tma_load_2d(dst + q * 2048, map, mn0 + 16 * q, k0, bar);
+    } else {
+        tma_load_2d(dst, map, k0, mn0, bar);
+    }
+}
+
+template <bool TA, bool TB>
+__global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_constant__ TmaBatch batch) {
+    constexpr bool A_MN = !TA;  // op(A) M x K: 'N' -> m contiguous
+    constexpr bool B_MN = TB;   // op(B) K x N: 'T' -> n contiguous
+    int q = 0;
+    const int bid = blockIdx.x;
+#pragma unroll 1
+    while (q + 1 < batch.n && bid >= batch.cta_start[q + 1]) ++q;
+    const TmaTask &t = batch.t[q];
+    const int local = bid - batch.cta_start[q];
+    const int tiles_m = (int)((t.M + BM - 1) / BM);
+    const int m0 = (local % tiles_m) * BM, n0 = (local / tiles_m) * BN;
+    const int64_t M = t.M, N = t.N;
+    const int tri = t.tri;
+    if ((tri == 1 && m0 + BM - 1 < n0) || (tri == 2 && n0 + BN - 1 < m0)) return;
+    const int KB = (int)((t.K + BK - 1) / BK);
+
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    // 1024-byte alignment of every stage (required by the 128-byte swizzle)
+    const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
+    unsigned char *sgen = smem_raw + (sbase - smem_u32(smem_raw));
+    const uint32_t bars = sbase + STAGES * STAGE_BYTES;  // full[STAGES], empty[STAGES]
+    auto full = [&](int s) { return bars + 8u * s; };
+    auto empty = [&](int s) { return bars + 8u * (STAGES + s); };
+
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(full(s), 1);
+            mbar_init(empty(s), NWARPS);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&t.mapA)) : "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&t.mapB)) : "memory");
+    }
+    __syncthreads();
+    auto produce = [&](int kb) {
+        const int s = kb % STAGES;
+        const uint32_t dst = sbase + s * STAGE_BYTES;
+        mbar_expect_tx(full(s), STAGE_BYTES);
+        issue_operand<A_MN, BM>(dst, &t.mapA, m0, kb * BK, full(s));
+        issue_operand<B_MN, BN>(dst + A_BYTES, &t.mapB, n0, kb * BK, full(s));
+    };
+    if (tid == 0)
+        for (int kb = 0; kb < STAGES - 1 && kb < KB; ++kb) produce(kb);
+
+    const int wm = (warp % NWM) * WM, wn = (warp / NWM) * WN;
+    const int fr = lane >> 2, fc = lane & 3;
+    constexpr int MF = WM / 8, NF = WN / 8;
+    // permuted k of this lane for step s: X[s] ^ Q[fc], X = {0,1,4,5}, Q = {0,3,12,15}
+    const int qk = (fc == 0) ? 0 : (fc == 1) ? 3 : (fc == 2) ? 12 : 15;
+    const uint32_t laneA = lane_part<A_MN>(fr, qk), laneB = lane_part<B_MN>(fr, qk);
+
+    double acc[MF][NF][2];
+#pragma unroll
+    for (int i = 0; i < MF; ++i)
+#pragma unroll
+        for (int j = 0; j < NF; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+    double fa[2][MF], fb[2][NF];
+    auto load_frags = [&](int buf, int stage, int s) {
+        const unsigned char *sa = sgen + stage * STAGE_BYTES;
+        const unsigned char *sb = sa + A_BYTES;
+        const int x = (s & 1) | ((s & 2) << 1);
+#pragma unroll
+        for (int i = 0; i < MF; ++i)
+            fa[buf][i] = *reinterpret_cast<const double *>(sa + (laneA ^ const_part<A_MN>(wm + i * 8, x)));
+#pragma unroll
+        for (int j = 0; j < NF; ++j)
+            fb[buf][j] = *reinterpret_cast<const double *>(sb + (laneB ^ const_part<B_MN>(wn + j * 8, x)));
+    };
+
+    mbar_wait(full(0), 0);
+    load_frags(0, 0, 0);
+#pragma unroll 1
+    for (int kb = 0; kb < KB; ++kb) {
+        const int st = kb % STAGES;
+#pragma unroll
+        for (int s = 0; s < BK / 4; ++s) {
+            const int cur = s & 1;
+            if (s + 1 < BK / 4) {
+                load_frags(cur ^ 1, st, s + 1);
+                if (s + 2 == BK / 4) {
+                    // last read of this stage issued: release it to the producer
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(empty(st));
+                }
+            } else if (kb + 1 < KB) {
+                const int nx = (kb + 1) % STAGES;
+                mbar_wait(full(nx), (uint32_t)(((kb + 1) / STAGES) & 1));
+                load_frags(cur ^ 1, nx, 0);
+            }
+#pragma unroll
+            for (int i = 0; i < MF; ++i)
+#pragma unroll
+                for (int j = 0; j < NF; ++j) dmma(acc[i][j], fa[cur][i], fb[cur][j]);
+        }
+        // producer: block kb + STAGES - 1 goes into the stage consumed at block kb - 1
+        if (tid == 0 && kb + STAGES - 1 < KB) {
+            if (kb >= 1) mbar_wait(empty((kb - 1) % STAGES), (uint32_t)(((kb - 1) / STAGES) & 1));
+            produce(kb + STAGES - 1);
+        }
+    }
+
+    // epilogue: D = alpha*acc + beta*C (C not read when beta == 0)
+    const double alpha = t.alpha, beta = t.beta;
+    double *C = t.C;
+    const int64_t ldc = t.ldc;
+#pragma unroll
+    for (int i = 0; i < MF; ++i) {
+        const int64_t r = m0 + wm + i * 8 + fr;
+        if (r >= M) continue;
+#pragma unroll
+        for (int j = 0; j < NF; ++j) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int64_t c = n0 + wn + j * 8 + fc * 2 + h;
+                if (c >= N) continue;
+                if ((tri == 1 && r < c) || (tri == 2 && r > c)) continue;
+                double *p = C + r + c * ldc;
+                double v = alpha * acc[i][j][h];
+                if (beta != 0.0) v = fma(beta, *p, v);
+                *p = v;
+            }
+        }
+    }
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                  const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                  const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+        cudaGetLastError();
+    }
+    return fn;
+}
+
+}  // namespace
+
+// Tensor map of a stored column-major operand (rows x cols, ld) for the TMA kernel.
+// mn_contig: the contiguous dimension is m/n (box 16 x 16); else it is k (box 16 x bmn).
+bool make_tma_operand(CUtensorMap *map, const double *X, int64_t rows, int64_t cols, int64_t ld,
+                      bool mn_contig, int bmn) {
+    EncodeTiledFn fn = encode_fn();
+    if (!fn) return false;
+    if (((uintptr_t)X & 15) || ((ld * 8) & 15) || rows <= 0 || cols <= 0) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * 8)};
+    cuuint32_t box[2] = {16u, mn_contig ? 16u : (cuuint32_t)bmn};
+    cuuint32_t estr[2] = {1u, 1u};
+    CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double *>(X), dims, strides, box,
+                    estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+int tma_bm() { return BM; }
+int tma_bn() { return BN; }
+
+cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st) {
+    if (b.n <= 0) return cudaSuccess;
+    constexpr size_t smem = STAGES * STAGE_BYTES + 2 * STAGES * 8 + 1024;
+    int total = 0;
+    for (int q = 0; q < b.n; ++q) {
+        b.cta_start[q] = total;
+        total += (int)(((b.t[q].M + BM - 1) / BM) * ((b.t[q].N + BN - 1) / BN));
+    }
+    b.cta_start[b.n] = total;
+    if (total == 0) return cudaSuccess;
+    static unsigned attr_set[4] = {0, 0, 0, 0};  // per (ta, tb) kernel, one bit per device
+    auto go = [&](void (*kern)(TmaBatch), int which) -> cudaError_t {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if (!(attr_set[which] & (1u << dev))) {
+            cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            if (e != cudaSuccess) return e;
+            attr_set[which] |= 1u << dev;
+        }
+        kern<<<total, NTHREADS, smem, st>>>(b);
+        return cudaGetLastError();
+    };
+    if (!ta && !tb) return go(dgemm_tma_kernel<false, false>, 0);
+    if (!ta && tb) return go(dgemm_tma_kernel<false, true>, 1);
+    if (ta && !tb) return go(dgemm_tma_kernel<true, false>, 2);
+    return go(dgemm_tma_kernel<true, true>, 3);
+}
+
+}  // namespace xk

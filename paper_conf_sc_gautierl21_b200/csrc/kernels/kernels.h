@@ -1,5 +1,6 @@
 // kernels.h -- internal launch interface of the sm_100a tile kernels (no torch types).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -24,6 +25,27 @@ struct TileBatch {
     int cta_start[kMaxBatch + 1] = {};
     TileTask t[kMaxBatch];
 };
+
+// TMA variant (dgemm_tma.cu): operands described by tensor maps (128-byte swizzle).
+struct TmaTask {
+    CUtensorMap mapA, mapB;  // stored A / B tiles (make_tma_operand)
+    double *C;
+    int64_t ldc, M, N, K;
+    double alpha, beta;
+    int tri;
+};
+constexpr int kMaxTmaBatch = 16;
+struct TmaBatch {
+    int n = 0;
+    int cta_start[kMaxTmaBatch + 1] = {};
+    TmaTask t[kMaxTmaBatch];
+};
+bool make_tma_operand(CUtensorMap *map, const double *X, int64_t rows, int64_t cols, int64_t ld,
+                      bool mn_contig, int bmn);
+int tma_bm();
+int tma_bn();
+cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st);
+bool tma_enabled();
 
 // All tasks of a batch share transA / transB (dgemm_tile.cu).
 cudaError_t launch_dgemm_batch(bool ta, bool tb, TileBatch &b, cudaStream_t st);
