@@ -7,8 +7,8 @@
 // address math, the per-k-block __syncthreads and cp.async waits (profiles/r01_*).  Here one
 // thread streams whole operand boxes with the Tensor Memory Accelerator
 // (cp.async.bulk.tensor.2d, zero-filled out of bounds so ragged tiles need no predication),
-// each stage completes on a transaction-count mbarrier, and warps release stages through an
-// "empty" mbarrier: no CTA-wide barrier in the main loop.
+// each stage completes on a transaction-count mbarrier, and the last warp to finish reading a
+// stage refills it (a shared-memory counter per stage): no CTA-wide barrier, no producer warp.
 //
 // Shared-memory layout: TMA 128-byte swizzle (16-byte chunk index XOR row % 8).  mn-contiguous
 // operands are loaded as 16(mn) x 16(k) boxes (rows = k), k-contiguous operands as one
@@ -120,15 +120,16 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
     // 1024-byte alignment of every stage (required by the 128-byte swizzle)
     const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
     unsigned char *sgen = smem_raw + (sbase - smem_u32(smem_raw));
-    const uint32_t bars = sbase + STAGES * STAGE_BYTES;  // full[STAGES], empty[STAGES]
+    const uint32_t bars = sbase + STAGES * STAGE_BYTES;  // full[STAGES] mbarriers
     auto full = [&](int s) { return bars + 8u * s; };
-    auto empty = [&](int s) { return bars + 8u * (STAGES + s); };
+    // per-stage count of warps done reading it; the last one refills the stage
+    int *done_cnt = reinterpret_cast<int *>(sgen + STAGES * STAGE_BYTES + 8 * STAGES);
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(full(s), 1);
-            mbar_init(empty(s), NWARPS);
+            done_cnt[s] = 0;
         }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&t.mapA)) : "memory");
@@ -143,7 +144,7 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
         issue_operand<B_MN, BN>(dst + A_BYTES, &t.mapB, n0, kb * BK, full(s));
     };
     if (tid == 0)
-        for (int kb = 0; kb < STAGES - 1 && kb < KB; ++kb) produce(kb);
+        for (int kb = 0; kb < STAGES && kb < KB; ++kb) produce(kb);
 
     const int wm = (warp % NWM) * WM, wn = (warp / NWM) * WN;
     const int fr = lane >> 2, fc = lane & 3;
@@ -181,9 +182,19 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
             if (s + 1 < BK / 4) {
                 load_frags(cur ^ 1, st, s + 1);
                 if (s + 2 == BK / 4) {
-                    // last read of this stage issued: release it to the producer
+                    // this warp's last read of the stage is done; the last warp to get here
+                    // refills the stage with block kb + STAGES (no CTA-wide barrier, no
+                    // dedicated producer warp)
                     __syncwarp();
-                    if (lane == 0) mbar_arrive(empty(st));
+                    if (lane == 0) {
+                        if (atomicAdd(&done_cnt[st], 1) == NWARPS - 1) {
+                            atomicExch(&done_cnt[st], 0);
+                            if (kb + STAGES < KB) {
+                                asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+                                produce(kb + STAGES);
+                            }
+                        }
+                    }
                 }
             } else if (kb + 1 < KB) {
                 const int nx = (kb + 1) % STAGES;
@@ -194,11 +205,6 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
             for (int i = 0; i < MF; ++i)
 #pragma unroll
                 for (int j = 0; j < NF; ++j) dmma(acc[i][j], fa[cur][i], fb[cur][j]);
-        }
-        // producer: block kb + STAGES - 1 goes into the stage consumed at block kb - 1
-        if (tid == 0 && kb + STAGES - 1 < KB) {
-            if (kb >= 1) mbar_wait(empty((kb - 1) % STAGES), (uint32_t)(((kb - 1) / STAGES) & 1));
-            produce(kb + STAGES - 1);
         }
     }
 
@@ -270,7 +276,7 @@ int tma_bn() { return BN; }
 
 cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st) {
     if (b.n <= 0) return cudaSuccess;
-    constexpr size_t smem = STAGES * STAGE_BYTES + 2 * STAGES * 8 + 1024;
+    constexpr size_t smem = STAGES * STAGE_BYTES + STAGES * 8 + STAGES * 4 + 1024;
     int total = 0;
     for (int q = 0; q < b.n; ++q) {
         b.cta_start[q] = total;
