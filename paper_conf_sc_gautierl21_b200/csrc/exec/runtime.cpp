@@ -458,7 +458,7 @@ int Runtime::issue(const Rec &R) {
         for (int q = 0; q < 4 && !conflict; ++q)
             if (r.dep[q] >= 0 && bt.contains_seq(r.dep[q])) conflict = true;
         if (conflict && (rc = flush_batch(g))) return rc;
-        bt.recs.push_back(&R);
+        bt.recs.push_back(R);
         bt.out_ids.push_back(idO);
         bt.in_ids.push_back(idA);
         bt.in_ids.push_back(idB);
@@ -506,7 +506,7 @@ int Runtime::flush_batch(int g) {
     tb.n = (int)bt.recs.size();
     int64_t flops = 0;
     for (int q = 0; q < tb.n; ++q) {
-        const Rec &R = *bt.recs[q];
+        const Rec &R = bt.recs[q];
         for (int j = 0; j < 4; ++j)
             if ((rc = wait_dep(s, R.r.dep[j]))) return rc;
         Buffer *O = buf(R.key, g, false, &rc);
@@ -535,7 +535,7 @@ int Runtime::flush_batch(int g) {
     Ev ev;
     if ((rc = record(s, g, &ev))) return rc;
     for (int q = 0; q < tb.n; ++q) {
-        const Rec &R = *bt.recs[q];
+        const Rec &R = bt.recs[q];
         seq_ev_[R.r.seq] = ev;
         Buffer *O = buf(R.key, g, false, &rc);
         O->writer = ev;
@@ -809,14 +809,15 @@ int Runtime::run(const xk_call_t &call, bool wait) {
     }
     std::vector<Rec> recs;
     std::string err;
-    rc = planner_->plan(call, recs, err);
+    size_t d2h0 = pending_d2h_.size();
+    // records are issued as the planner produces them: the GPUs start on the first copies
+    // and tasks while the rest of the call is still being planned
+    Planner::Sink sink = [this](const Rec &r) { return issue(r); };
+    rc = planner_->plan(call, recs, err, &sink);
     if (rc) {
-        set_error(err);
+        if (rc != XK_ERR_CUDA && rc != XK_ERR_OOM) set_error(err);
         return rc;
     }
-    size_t d2h0 = pending_d2h_.size();
-    for (const Rec &r : recs)
-        if ((rc = issue(r))) return rc;
     for (size_t g = 0; g < batch_.size(); ++g)
         if ((rc = flush_batch((int)g))) return rc;
     if (call.routine <= XK_ROUTINE_DTRSM && call.sync) {

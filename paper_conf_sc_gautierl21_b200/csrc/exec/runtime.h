@@ -38,12 +38,12 @@ struct Buffer {
 
 // Tile tasks of one GPU waiting to be launched together (grouped GEMM launch).
 struct PendingBatch {
-    std::vector<const Rec *> recs;
+    std::vector<Rec> recs;  // copies (records are issued while they are planned)
     std::vector<int64_t> out_ids, in_ids;  // buffer ids written / read
     char ta = 'N', tb = 'N';
     bool contains_seq(int64_t seq) const {
-        for (const Rec *r : recs)
-            if (r->r.seq == seq) return true;
+        for (const Rec &r : recs)
+            if (r.r.seq == seq) return true;
         return false;
     }
     bool touches(int64_t id, bool write) const {

@@ -118,10 +118,7 @@ int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t
 }
 
 int Planner::key_of(int mat, int64_t bi, int64_t bj) {
-    std::string k(sizeof(int) + 2 * sizeof(int64_t), '\0');
-    std::memcpy(&k[0], &mat, sizeof(int));
-    std::memcpy(&k[sizeof(int)], &bi, sizeof(int64_t));
-    std::memcpy(&k[sizeof(int) + sizeof(int64_t)], &bj, sizeof(int64_t));
+    const uint64_t k = tile_key(mat, bi, bj);
     auto it = keymap_.find(k);
     if (it != keymap_.end()) return it->second;
     Entry e;
@@ -144,7 +141,15 @@ int Planner::key_of(int mat, int64_t bi, int64_t bj) {
 // step 4: source selection for a tile needed on GPU d at request time treq.
 int Planner::select_source(const Entry &e, int64_t ver, int d, int64_t treq, int *state) const {
     const int G = topo_.G;
-    std::vector<int> V, I;
+    struct Small {  // G <= XK_MAX_GPUS candidates, no allocation
+        int v[XK_MAX_GPUS];
+        int n = 0;
+        void push_back(int g) { v[n++] = g; }
+        bool empty() const { return n == 0; }
+        int front() const { return v[0]; }
+        const int *begin() const { return v; }
+        const int *end() const { return v + n; }
+    } V, I;
     for (int g = 0; g < G; ++g) {
         if (g == d) continue;
         const NodeCopy &c = e.gpu[g];
@@ -152,7 +157,7 @@ int Planner::select_source(const Entry &e, int64_t ver, int d, int64_t treq, int
         if (c.t_done <= treq) V.push_back(g); else I.push_back(g);
     }
     bool host_ok = e.host.present && e.host.ver == ver;
-    auto ranked_best = [&](const std::vector<int> &L) {
+    auto ranked_best = [&](const Small &L) {
         int best = -1;
         std::tuple<int, int, int> bk;
         for (int g : L) {
@@ -162,7 +167,7 @@ int Planner::select_source(const Entry &e, int64_t ver, int d, int64_t treq, int
         }
         return best;
     };
-    auto lowest = [&](const std::vector<int> &L) { return L.empty() ? -1 : L.front(); };
+    auto lowest = [&](const Small &L) { return L.empty() ? -1 : L.front(); };
     int mode = flags_.topo;
     if (mode == XK_TOPO_HOME) {
         if (host_ok) { *state = XK_SRC_HOST; return XK_HOST; }
@@ -171,7 +176,7 @@ int Planner::select_source(const Entry &e, int64_t ver, int d, int64_t treq, int
         *state = XK_SRC_NONE;
         return -2;
     }
-    auto pick = [&](const std::vector<int> &L) {
+    auto pick = [&](const Small &L) {
         return mode == XK_TOPO_RANKED ? ranked_best(L) : lowest(L);
     };
     if (!V.empty()) { *state = XK_SRC_VALID; return pick(V); }
@@ -228,7 +233,7 @@ bool Planner::emit_copy(int key, int64_t ver, int d, int64_t treq, int operand,
     R.key = key;
     R.sub_rows = e.rows;
     R.sub_cols = e.cols;
-    out.push_back(R);
+    emit(R, out);
     NodeCopy &c = e.gpu[d];
     c.present = true;
     c.ver = ver;
@@ -271,7 +276,7 @@ void Planner::emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, i
     R.sub_c0 = c0;
     R.sub_rows = rows;
     R.sub_cols = cols;
-    out.push_back(R);
+    emit(R, out);
     if (r0 == 0 && c0 == 0 && rows == e.rows && cols == e.cols) {
         e.host.present = true;
         e.host.ver = e.ver;
@@ -288,14 +293,42 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
     const int G = topo_.G;
     const int W = std::max(1, flags_.window);
     // pending reads per (key, version) in this call; last writer per output tile
-    std::map<std::pair<int, int64_t>, int64_t> readers;
-    std::map<int, size_t> last;
+    struct PairHash {
+        size_t operator()(const std::pair<int, int64_t> &p) const {
+            return std::hash<uint64_t>()(((uint64_t)p.first << 32) ^ (uint64_t)p.second * 0x9E3779B97F4A7C15ULL);
+        }
+    };
+    // pending reads per (key, version) in this call, resolved once to flat counter slots
+    std::vector<int64_t> pending;
+    {
+        std::unordered_map<std::pair<int, int64_t>, int, PairHash> slot;
+        slot.reserve(tasks.size() * 2 + 16);
+        auto slot_of = [&](int key, int64_t ver) {
+            auto it = slot.find({key, ver});
+            if (it != slot.end()) return it->second;
+            int id = (int)pending.size();
+            pending.push_back(0);
+            slot.emplace(std::make_pair(key, ver), id);
+            return id;
+        };
+        for (auto &t : tasks)
+            for (auto &in : t.in) {
+                in.cnt = slot_of(in.key, in.ver);
+                pending[in.cnt]++;
+            }
+        for (auto &t : tasks) {
+            auto it = slot.find({t.out_key, t.out_ver - 1});
+            t.war = (it == slot.end()) ? -1 : it->second;
+        }
+    }
+    // last writer per output tile
+    std::unordered_map<int, size_t> last;
     for (size_t q = 0; q < tasks.size(); ++q) {
-        for (auto &in : tasks[q].in) readers[{in.key, in.ver}]++;
         auto it = last.find(tasks[q].out_key);
         if (it == last.end() || tasks[it->second].out_ver < tasks[q].out_ver) last[tasks[q].out_key] = q;
     }
     for (auto &kv : last) tasks[kv.second].last_writer = true;
+    out.reserve(out.size() + tasks.size() * 2);
     std::vector<std::vector<int>> lists(G);
     for (size_t q = 0; q < tasks.size(); ++q) lists[tasks[q].gpu].push_back((int)q);
     for (int d = 0; d < G; ++d) {
@@ -312,23 +345,32 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
             if (entries_[in.key].ver != in.ver) return false;
         const Entry &o = entries_[t.out_key];
         if (o.ver != t.out_ver - 1) return false;
-        auto it = readers.find({t.out_key, t.out_ver - 1});
-        int64_t pend = (it == readers.end()) ? 0 : it->second;
+        int64_t pend = (t.war < 0) ? 0 : pending[t.war];
         for (auto &in : t.in)
             if (in.key == t.out_key && in.ver == t.out_ver - 1) pend--;
         return pend == 0;
     };
     size_t done = 0;
+    std::vector<std::pair<int64_t, int>> cand(G);
     while (done < tasks.size()) {
-        int best = -1;
-        int64_t best_treq = 0;
+        // the GPU with the smallest request time whose next task is ready (ties: lower id);
+        // readiness is only evaluated in (treq, d) order until the first ready one
+        int nc = 0;
         for (int d = 0; d < G; ++d) {
             if (pos[d] == lists[d].size()) continue;
-            const Task &t = tasks[lists[d][pos[d]]];
-            if (!ready(t)) continue;
             const auto &h = ends_[d];
             int64_t treq = (int64_t)h.size() >= W ? h[h.size() - W] : 0;
-            if (best < 0 || treq < best_treq) { best = d; best_treq = treq; }
+            cand[nc++] = {treq, d};
+        }
+        std::sort(cand.begin(), cand.begin() + nc);
+        int best = -1;
+        int64_t best_treq = 0;
+        for (int c = 0; c < nc; ++c) {
+            if (ready(tasks[lists[cand[c].second][pos[cand[c].second]]])) {
+                best = cand[c].second;
+                best_treq = cand[c].first;
+                break;
+            }
         }
         if (best < 0) {
             err = "planner deadlock: no ready task (output aliases an input?)";
@@ -349,7 +391,7 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
             }
             in_ready = std::max(in_ready, e.gpu[d].t_done);
             if (p < 4) deps[p] = e.gpu[d].producer;
-            readers[{in.key, in.ver}]--;
+            pending[in.cnt]--;
         }
         int64_t t0 = std::max(gpu_free_[d], in_ready);
         int64_t t1 = t0 + dur(t.flops, topo_.rate_mflops);
@@ -389,7 +431,11 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
         R.m = t.m;
         R.n = t.n;
         R.k = t.k;
-        out.push_back(R);
+        emit(R, out);
+        if (sink_rc_) {
+            err = "issue failed";
+            return sink_rc_;
+        }
         o.ver = t.out_ver;
         for (int g = 0; g < G; ++g)
             if (g != d) o.gpu[g].present = false;
@@ -429,6 +475,7 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
     Versions V;
     V.e = &entries_;
     std::vector<Task> tasks;
+    tasks.reserve((size_t)(tm * tn * std::max<int64_t>(tkn, 1)));
     for (int64_t j = 0; j < tn; ++j) {
         for (int64_t i = 0; i < tm; ++i) {
             int keyC = key_of(mc, i, j);
@@ -472,7 +519,11 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                 t.i = i; t.j = j;
                 t.m = mt; t.n = nt; t.k = kt;
                 t.flops = 2 * mt * nt * kt;
-                int64_t sk[5] = {kk, (i + j + kk) % tmod, i, j, 0};
+                // staggered k-chains (reading Q12'): tile (i,j) starts its chain at slot
+                // (i+j) mod tk, so chains begin and end at different times -- C's H2D spreads
+                // over the first tk slots and its D2H over the last ones instead of piling up
+                // at k = 0 and at the end
+                int64_t sk[5] = {kk + (i + j) % tkn, (i + j + kk) % tmod, i, j, 0};
                 std::copy(sk, sk + 5, t.skey);
                 tasks.push_back(t);
             }
@@ -863,11 +914,7 @@ int Planner::plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::strin
     int64_t rend = std::min(M.rows, r0 + c.m), cend = std::min(M.cols, c0 + c.n);
     for (int64_t bj = c0 / T; bj * T < cend; ++bj) {
         for (int64_t bi = r0 / T; bi * T < rend; ++bi) {
-            std::string k(sizeof(int) + 2 * sizeof(int64_t), '\0');
-            std::memcpy(&k[0], &mat, sizeof(int));
-            std::memcpy(&k[sizeof(int)], &bi, sizeof(int64_t));
-            std::memcpy(&k[sizeof(int) + sizeof(int64_t)], &bj, sizeof(int64_t));
-            auto it = keymap_.find(k);
+            auto it = keymap_.find(tile_key(mat, bi, bj));
             if (it == keymap_.end()) continue;
             Entry &e = entries_[it->second];
             if (e.host.present && e.host.ver == e.ver) continue;  // host already valid
@@ -962,7 +1009,25 @@ void Planner::finish_call(const xk_call_t &c) {
     }
 }
 
-int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
+void Planner::emit(const Rec &R, std::vector<Rec> &out) {
+    if (!sink_) {
+        out.push_back(R);
+        return;
+    }
+    if (sink_rc_) return;  // an earlier record failed to issue: stop
+    sink_rc_ = (*sink_)(R);
+}
+
+int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err, const Sink *sink) {
+    sink_ = sink;
+    sink_rc_ = 0;
+    int rc = plan_impl(c, out, err);
+    sink_ = nullptr;
+    if (rc == XK_OK && sink_rc_) rc = sink_rc_;
+    return rc;
+}
+
+int Planner::plan_impl(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
     int rc;
     switch (c.routine) {
     case XK_ROUTINE_DGEMM:

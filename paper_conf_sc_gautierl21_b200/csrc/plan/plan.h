@@ -10,6 +10,7 @@
 // Readings are listed in DESIGN.md.
 #pragma once
 #include <cstdint>
+#include <functional>
 #include <string>
 #include <unordered_map>
 #include <vector>
@@ -76,8 +77,11 @@ class Planner {
 public:
     Planner(const Topology &t, const Flags &f);
 
-    // Plan one call; appends records to out.  Returns 0 or XK_ERR_*.
-    int plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
+    // Plan one call.  Records go to `sink` as they are produced (the executor issues them
+    // while planning continues -- the GPUs start on the first records) or, without a sink,
+    // are appended to out.  Returns 0 or XK_ERR_* (a sink error aborts the plan).
+    using Sink = std::function<int(const Rec &)>;
+    int plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err, const Sink *sink = nullptr);
 
     // Full synchronisation point (return of a sync routine, xk_sync): every copy is
     // complete, clocks restart at 0.
@@ -95,13 +99,26 @@ public:
     int link_class(int s, int d) const { return cls_[(size_t)s * (topo_.G + 1) + d]; }
 
 private:
-    struct Input { int key; int64_t ver; int operand; };
+    struct Input { int key; int64_t ver; int operand; int cnt = -1; };  // cnt: readers slot
+    struct Inputs {  // at most 4 inputs per task, no heap allocation
+        Input v[4];
+        int n = 0;
+        void push_back(const Input &x) { v[n++] = x; }
+        size_t size() const { return (size_t)n; }
+        Input &operator[](size_t i) { return v[i]; }
+        const Input &operator[](size_t i) const { return v[i]; }
+        Input *begin() { return v; }
+        Input *end() { return v + n; }
+        const Input *begin() const { return v; }
+        const Input *end() const { return v + n; }
+    };
     struct Task {
         int gpu = 0;
         int op = XK_OP_GEMM;
         int out_key = -1;
         int64_t out_ver = 0;        // version produced
-        std::vector<Input> in;      // inputs in position order (deps follow this order)
+        Inputs in;                  // inputs in position order (deps follow this order)
+        int war = -1;               // readers slot of (out_key, out_ver - 1)
         int keyA = -1, keyB = -1;   // kernel roles
         char ta = 'N', tb = 'N', side = 'L', uplo = 'L', diag = 'N';
         int tri = 0;
@@ -121,8 +138,15 @@ private:
         int64_t bump(int key) { int64_t v = get(key) + 1; cur[key] = v; return v; }
     };
 
+    int plan_impl(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
+    void emit(const Rec &R, std::vector<Rec> &out);
+    const Sink *sink_ = nullptr;
+    int sink_rc_ = 0;
     int find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t cols, std::string &err);
     int key_of(int mat, int64_t bi, int64_t bj);
+    static uint64_t tile_key(int mat, int64_t bi, int64_t bj) {
+        return ((uint64_t)mat << 48) | ((uint64_t)bi << 24) | (uint64_t)bj;  // < 2^24 tiles per dim
+    }
     int64_t dur(int64_t amount, int64_t rate) const;  // ceil(amount*1000/rate) ns
     int select_source(const Entry &e, int64_t ver, int d, int64_t treq, int *state) const;
     bool emit_copy(int key, int64_t ver, int d, int64_t treq, int operand, std::vector<Rec> &out);
@@ -143,7 +167,7 @@ private:
     std::vector<int> cls_;
     std::vector<Matrix> mats_;
     std::vector<Entry> entries_;
-    std::unordered_map<std::string, int> keymap_;
+    std::unordered_map<uint64_t, int> keymap_;  // (mat, bi, bj) packed, see tile_key()
     std::vector<int64_t> link_free_;     // (G+1)^2
     std::vector<int64_t> gpu_free_;      // G
     std::vector<std::vector<int64_t>> ends_;  // per GPU task end-time history (since last sync)

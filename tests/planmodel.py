@@ -245,7 +245,7 @@ class Model:
                     at = self.tile(A, lda, kk, i) if ta else self.tile(A, lda, i, kk)
                     bt = self.tile(B, ldb, j, kk) if tb else self.tile(B, ldb, kk, j)
                     ins = [(at, 0), (bt, 1)] + ([(ct, 2)] if (kk > 0 or beta != 0) else [])
-                    tasks.append(self._task(vers, OP_GEMM, i, j, ct, ins, (kk, (i + j + kk) % tmod, i, j, 0),
+                    tasks.append(self._task(vers, OP_GEMM, i, j, ct, ins, (kk + (i + j) % tk, (i + j + kk) % tmod, i, j, 0),
                                             2 * mt * nt * kt, kk))
         return tasks
 
