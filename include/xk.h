@@ -174,12 +174,20 @@ typedef struct xk_stats {
     double kernel_ms_total;          /* summed tile-kernel launch time (when timing on) */
     int64_t kernel_timed_launches;   /* launches included in kernel_ms_total */
     int64_t kernel_timed_flops;      /* algorithmic flops of those launches (2*m*n*k per task) */
+    double trace_ms[4];              /* with tracing on: summed op time by kind
+                                        [H2D, P2P, kernel, D2H] (paper Fig. 6 breakdown) */
 } xk_stats_t;
 int xk_get_stats(xk_stats_t *out);
 int xk_reset_stats(void);
 /* 1 = time every tile-kernel launch with CUDA events (bench roofline); grouped launches are
  * then serialised on one kernel stream per GPU so each duration is its own.  0 = off. */
 int xk_set_kernel_timing(int on);
+/* Timeline tracing (paper: nvprof Gantt charts).  path != NULL: record
+ * every copy and kernel launch with CUDA events from now on; path == NULL: stop and write the
+ * Chrome-trace JSON (chrome://tracing / Perfetto) of everything recorded since to the path
+ * given at start.  Waits for pending work.  XK_TRACE=path in the environment traces the whole
+ * session and writes it at xk_finalize. */
+int xk_trace(const char *path);
 
 /* (G+1) x (G+1) link matrix in MB/s, row = source, column = destination, index G =
  * host; diagonal = device-local copy bandwidth.  Filled by xk_init (probe or defaults). */

@@ -168,7 +168,13 @@ def get_stats():
     for f in ("forwards_inflight", "forwards_valid", "kernel_launches", "host_registrations",
               "kernel_ms_total", "kernel_timed_launches", "kernel_timed_flops"):
         out[f] = getattr(st, f)
+    out["trace_ms"] = dict(zip(("h2d", "p2p", "kernel", "d2h"), list(st.trace_ms)))
     return out
+
+
+def trace(path):
+    """Start (path) or stop and write (None) the Chrome-trace timeline."""
+    return _check(lib().xk_trace(path.encode() if path else None))
 
 
 def reset_stats():

@@ -46,7 +46,8 @@ class Stats(ctypes.Structure):
                 ("tasks", i64 * MAX_GPUS), ("flops", i64 * MAX_GPUS),
                 ("forwards_inflight", i64), ("forwards_valid", i64), ("kernel_launches", i64),
                 ("host_registrations", i64), ("kernel_ms_total", c_double),
-                ("kernel_timed_launches", i64), ("kernel_timed_flops", i64)]
+                ("kernel_timed_launches", i64), ("kernel_timed_flops", i64),
+                ("trace_ms", c_double * 4)]
 
 
 class Topo(ctypes.Structure):
@@ -116,6 +117,7 @@ _SIGS = [
     ("xk_reset_stats", c_int, []),
     ("xk_set_kernel_timing", c_int, [c_int]),
     ("xk_get_topology", c_int, [ctypes.POINTER(Topo)]),
+    ("xk_trace", c_int, [ctypes.c_char_p]),
     ("xk_plan_session_create", c_int, [ctypes.POINTER(Topo), ctypes.POINTER(Flags), ctypes.POINTER(vp)]),
     ("xk_plan_session_call", c_int, [vp, ctypes.POINTER(Call), ctypes.POINTER(PlanRec), i64,
                                      ctypes.POINTER(i64)]),

@@ -384,6 +384,13 @@ int xk_set_kernel_timing(int on) {
     rt->kernel_timing = on != 0;
     return XK_OK;
 }
+int xk_trace(const char *path) {
+    xk::Runtime *rt = runtime();
+    if (!rt) return need_init();
+    if (path) return rt->trace_start(path);
+    return rt->trace_stop();
+}
+
 int xk_get_topology(xk_topo_t *out) {
     xk::Runtime *rt = runtime();
     if (!rt) return need_init();

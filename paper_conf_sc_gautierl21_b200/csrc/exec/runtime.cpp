@@ -139,6 +139,8 @@ int Runtime::init(const xk_config_t &cfg) {
     planner_.reset(new Planner(topo, flags_));
     std::memset(&stats, 0, sizeof(stats));
     stats.ngpus = G;
+    const char *tp = std::getenv("XK_TRACE");
+    if (tp && *tp) return trace_start(tp);
     return XK_OK;
 }
 
@@ -351,7 +353,10 @@ int Runtime::issue(const Rec &R) {
             if ((rc = wait_on(s, rd))) return rc;
         if ((rc = wait_on(s, B->writer))) return rc;
         const char *host = (const char *)(uintptr_t)M.base + (e.bi * T + e.bj * T * M.ld) * 8;
+        cudaEvent_t ta = nullptr;
+        if (tracing_ && (rc = trace_begin(g, s, &ta))) return rc;
         if ((rc = copy_host(true, B->p, B->ld, (char *)host, M.ld, e.rows, e.cols, s))) return rc;
+        if (tracing_) trace_end(g, s, ta, 0, "H2D", r.work);
         Ev ev;
         if ((rc = record(s, g, &ev))) return rc;
         seq_ev_[r.seq] = ev;
@@ -375,7 +380,10 @@ int Runtime::issue(const Rec &R) {
             if ((rc = wait_on(s, rd))) return rc;
         if ((rc = wait_on(s, D->writer))) return rc;
         // store-and-forward of a whole compact tile over NVLink (copy engine, SMs stay free)
+        cudaEvent_t ta = nullptr;
+        if (tracing_ && (rc = trace_begin(g, s, &ta))) return rc;
         XK_CK(cudaMemcpyAsync(D->p, S->p, S->bytes, cudaMemcpyDeviceToDevice, s));
+        if (tracing_) trace_end(g, s, ta, 1, r.src_state == XK_SRC_INFLIGHT ? "P2P fwd-inflight" : "P2P", r.work);
         Ev ev;
         if ((rc = record(s, g, &ev))) return rc;
         seq_ev_[r.seq] = ev;
@@ -411,6 +419,8 @@ int Runtime::issue(const Rec &R) {
             if (R.keyB >= 0 && !(B = buf(R.keyB, g, false, &rc))) return rc;
             O = buf(R.key, g, false, &rc);
             cudaError_t ke = cudaSuccess;
+            cudaEvent_t ta = nullptr;
+            if (tracing_ && (rc = trace_begin(g, s, &ta))) return rc;
             if (R.op == XK_OP_SCALE) {
                 ke = launch_scale_tri(R.m, R.n, R.beta, O->p, O->ld, R.tri, s);
             } else if (R.op == XK_OP_TRSM_DIAG || R.op == XK_OP_TRMM_DIAG) {
@@ -437,6 +447,10 @@ int Runtime::issue(const Rec &R) {
                 return XK_ERR_INTERNAL;
             }
             if (ke != cudaSuccess) return cuda_fail(ke, "tile kernel launch");
+            if (tracing_) {
+                static const char *nm[] = {"gemm", "scale", "gemm_tri", "symm_diag", "trmm_diag", "trsm_diag"};
+                trace_end(g, s, ta, 2, nm[R.op], r.work);
+            }
             Ev ev;
             if ((rc = record(s, g, &ev))) return rc;
             seq_ev_[r.seq] = ev;
@@ -477,7 +491,10 @@ int Runtime::issue(const Rec &R) {
         char *host = (char *)(uintptr_t)M.base +
                      ((e.bi * T + R.sub_r0) + (e.bj * T + R.sub_c0) * M.ld) * 8;
         const double *src = S->p + R.sub_r0 + R.sub_c0 * S->ld;
+        cudaEvent_t ta = nullptr;
+        if (tracing_ && (rc = trace_begin(gs, s, &ta))) return rc;
         if ((rc = copy_host(false, (double *)src, S->ld, host, M.ld, R.sub_rows, R.sub_cols, s))) return rc;
+        if (tracing_) trace_end(gs, s, ta, 3, "D2H", r.work);
         Ev ev;
         if ((rc = record(s, gs, &ev))) return rc;
         seq_ev_[r.seq] = ev;
@@ -525,8 +542,11 @@ int Runtime::flush_batch(int g) {
         XK_CK(cudaEventCreate(&t1));
         XK_CK(cudaEventRecord(t0, s));
     }
+    cudaEvent_t tra = nullptr;
+    if (tracing_ && (rc = trace_begin(g, s, &tra))) return rc;
     cudaError_t ke = launch_dgemm_batch(bt.ta == 'T', bt.tb == 'T', tb, s);
     if (ke != cudaSuccess) return cuda_fail(ke, "tile kernel launch");
+    if (tracing_) trace_end(g, s, tra, 2, "gemm batch x" + std::to_string(tb.n), flops);
     if (kernel_timing) {
         XK_CK(cudaEventRecord(t1, s));
         ktimers_.push_back({t0, t1});
@@ -570,6 +590,84 @@ int Runtime::flush_for(const Rec &R) {
         }
     }
     return XK_OK;
+}
+
+// ---------------------------------------------------------------- timeline tracing
+int Runtime::trace_begin(int g, cudaStream_t s, cudaEvent_t *a) {
+    XK_CK(cudaEventCreate(a));
+    XK_CK(cudaEventRecord(*a, s));
+    (void)g;
+    return XK_OK;
+}
+
+void Runtime::trace_end(int g, cudaStream_t s, cudaEvent_t a, int kind, std::string name, int64_t work) {
+    cudaEvent_t b = nullptr;
+    if (cudaEventCreate(&b) != cudaSuccess || cudaEventRecord(b, s) != cudaSuccess) {
+        cudaGetLastError();
+        return;
+    }
+    trace_ops_.push_back({g, kind, a, b, std::move(name), work});
+}
+
+// After a full sync: turn the recorded event pairs into Chrome-trace events.
+void Runtime::trace_collect() {
+    static const char *tid[] = {"H2D", "P2P-in", "kernels", "D2H"};
+    for (auto &op : trace_ops_) {
+        float t0 = 0, t1 = 0;
+        if (cudaEventElapsedTime(&t0, trace_base_[op.g], op.a) == cudaSuccess &&
+            cudaEventElapsedTime(&t1, trace_base_[op.g], op.b) == cudaSuccess) {
+            char buf[256];
+            snprintf(buf, sizeof buf,
+                     "{\"name\":\"%s\",\"ph\":\"X\",\"ts\":%.3f,\"dur\":%.3f,\"pid\":\"GPU %d\",\"tid\":\"%s\",\"args\":{\"%s\":%lld}}",
+                     op.name.c_str(), t0 * 1e3, (t1 - t0) * 1e3, op.g, tid[op.kind],
+                     op.kind == 2 ? "flops" : "bytes", (long long)op.work);
+            trace_json_.push_back(buf);
+            stats.trace_ms[op.kind] += (t1 - t0);
+        }
+        cudaEventDestroy(op.a);
+        cudaEventDestroy(op.b);
+    }
+    cudaGetLastError();
+    trace_ops_.clear();
+}
+
+int Runtime::trace_start(const std::string &path) {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    int rc = sync_all();
+    if (rc) return rc;
+    trace_path_ = path;
+    trace_json_.clear();
+    trace_base_.assign(devs_.size(), nullptr);
+    for (size_t g = 0; g < devs_.size(); ++g) {
+        XK_CK(cudaSetDevice(devs_[g].phys));
+        XK_CK(cudaEventCreate(&trace_base_[g]));
+        XK_CK(cudaEventRecord(trace_base_[g], devs_[g].h2d));
+    }
+    cur_dev_ = -1;
+    tracing_ = true;
+    return XK_OK;
+}
+
+int Runtime::trace_stop() {
+    std::lock_guard<std::recursive_mutex> lk(mu);
+    if (!tracing_) return XK_OK;
+    int rc = sync_all();  // collects the remaining ops
+    tracing_ = false;
+    FILE *f = fopen(trace_path_.c_str(), "w");
+    if (f) {
+        fprintf(f, "{\"traceEvents\":[\n");
+        for (size_t i = 0; i < trace_json_.size(); ++i)
+            fprintf(f, "%s%s\n", trace_json_[i].c_str(), i + 1 < trace_json_.size() ? "," : "");
+        fprintf(f, "],\"displayTimeUnit\":\"ms\"}\n");
+        fclose(f);
+    } else if (!rc) {
+        set_error("xk_trace: cannot write " + trace_path_);
+        rc = XK_ERR_CONFIG;
+    }
+    for (cudaEvent_t e : trace_base_) cudaEventDestroy(e);
+    trace_base_.clear();
+    trace_json_.clear();
+    return rc;
 }
 
 // Boundaries of host registrations strictly inside [lo, hi): a pinned copy must not
@@ -735,6 +833,7 @@ int Runtime::sync_all() {
         XK_CK(cudaStreamSynchronize(d.d2h));
     }
     cur_dev_ = -1;
+    if (tracing_) trace_collect();
     for (size_t q = 0; q < ktimers_.size(); ++q) {
         float ms = 0;
         if (cudaEventElapsedTime(&ms, ktimers_[q].first, ktimers_[q].second) == cudaSuccess) {
@@ -848,6 +947,7 @@ int Runtime::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
 
 int Runtime::finalize() {
     std::lock_guard<std::recursive_mutex> lk(mu);
+    if (tracing_) trace_stop();
     int rc = sync_all();
     for (size_t g = 0; g < devs_.size(); ++g) {
         Device &d = devs_[g];

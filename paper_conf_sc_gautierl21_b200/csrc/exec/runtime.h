@@ -85,6 +85,9 @@ public:
 
     xk_stats_t stats{};
     bool kernel_timing = false;
+    // ---- timeline tracing
+    int trace_start(const std::string &path);
+    int trace_stop();
     Topology topo;
     std::vector<int> perf_rank;
     std::recursive_mutex mu;
@@ -119,7 +122,21 @@ private:
     std::vector<Ev> pending_d2h_;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ktimers_;
     std::vector<int64_t> ktimer_flops_;
-    std::vector<std::pair<int, std::pair<double *, size_t>>> scratch_;  // freed at the next full sync
+    std::vector<std::pair<int, std::pair<double *, size_t>>> scratch_;
+    struct TraceOp {
+        int g, kind;  // kind 0 H2D, 1 P2P, 2 kernel, 3 D2H
+        cudaEvent_t a, b;
+        std::string name;
+        int64_t work;
+    };
+    bool tracing_ = false;
+    std::string trace_path_;
+    std::vector<cudaEvent_t> trace_base_;  // per logical GPU
+    std::vector<TraceOp> trace_ops_;
+    std::vector<std::string> trace_json_;
+    int trace_begin(int g, cudaStream_t s, cudaEvent_t *a);
+    void trace_end(int g, cudaStream_t s, cudaEvent_t a, int kind, std::string name, int64_t work);
+    void trace_collect();  // freed at the next full sync
     std::map<uintptr_t, size_t> registered_;    // user-registered host ranges
     std::map<uintptr_t, size_t> internal_reg_;  // registered by the library on first use
     int cur_dev_ = -1;

@@ -220,3 +220,31 @@ def test_full_size_n32768_sampled():
     ref = oracle.dgemm_sampled("N", "N", N, 1.5, A, B, -0.75, C0[ii, jj], ii, jj)
     mag = 1.5 * np.einsum("qk,kq->q", np.abs(A[ii, :]), np.abs(B[:, jj])) + 0.75 * np.abs(C0[ii, jj])
     assert np.all(np.abs(C[ii, jj] - ref) <= 4 * N * 2.0 ** -53 * mag)
+
+
+def test_trace_timeline(tmp_path):
+    """xk_trace: every copy and kernel launch appears in the Chrome trace with its bytes /
+    flops; the per-kind byte totals equal the executor's counters (paper Fig. 6 breakdown)."""
+    import json
+    G, T, N = 2, 128, 384
+    A, B, C = inputs.uniform(1, N, N), inputs.uniform(2, N, N), inputs.uniform(3, N, N)
+    logical(G, tile=T)
+    try:
+        path = str(tmp_path / "trace.json")
+        xk.reset_stats()
+        xk.trace(path)
+        xk.dgemm("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
+        xk.trace(None)
+        st = xk.get_stats()
+    finally:
+        xk.finalize()
+    ev = json.load(open(path))["traceEvents"]
+    by = {}
+    for e in ev:
+        by.setdefault(e["tid"], 0)
+        by[e["tid"]] += e["args"].get("bytes", 0)
+        assert e["dur"] >= 0
+    assert by["H2D"] == sum(st["h2d_bytes"]) and by["D2H"] == sum(st["d2h_bytes"])
+    assert by["P2P-in"] == sum(st["p2p_in_bytes"]) > 0
+    assert any(e["tid"] == "kernels" for e in ev)
+    assert st["trace_ms"]["kernel"] > 0 and st["trace_ms"]["h2d"] > 0
