@@ -60,16 +60,22 @@ def parse():
 
 
 # --------------------------------------------------------------------------- distributed
-def dist_setup():
+def dist_setup(backend=None):
+    """One process per GPU under torchrun (RANK/LOCAL_RANK/WORLD_SIZE/MASTER_* from the env).
+    backend: "nccl" on GPU boxes (default), "gloo" for the CPU tests of this path."""
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     if ws > 1:
         import torch
         import torch.distributed as dist
-        lr = int(os.environ.get("LOCAL_RANK", rank))
-        torch.cuda.set_device(lr)
+        backend = backend or os.environ.get("XK_DIST_BACKEND", "nccl")
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+        if backend == "nccl":
+            lr = int(os.environ.get("LOCAL_RANK", rank))
+            torch.cuda.set_device(lr)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+        else:
+            dist.init_process_group(backend)
     return rank, ws
 
 
@@ -80,11 +86,14 @@ def barrier(ws):
 
 
 def max_over_ranks(x, ws):
+    """Timing is taken as the max over ranks (every rank measured the same barrier-bracketed
+    interval; rank 0 drove all GPUs)."""
     if ws == 1:
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
