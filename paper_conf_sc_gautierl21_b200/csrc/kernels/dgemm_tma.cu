@@ -110,7 +110,15 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
     const TmaTask &t = batch.t[q];
     const int local = bid - batch.cta_start[q];
     const int tiles_m = (int)((t.M + BM - 1) / BM);
-    const int m0 = (local % tiles_m) * BM, n0 = (local / tiles_m) * BN;
+    // grouped raster: CTAs run GROUP_M m-blocks at a time across all n-blocks, so the CTAs
+    // resident together share A and B slabs in L2 instead of streaming all of A per column
+    const int tiles_n = (int)((t.N + BN - 1) / BN);
+    const int gm = batch.group_m > 0 ? batch.group_m : tiles_m;
+    const int per_group = gm * tiles_n;
+    const int first = (local / per_group) * gm;
+    const int gsz = min(tiles_m - first, gm);
+    const int in_group = local % per_group;
+    const int m0 = (first + in_group % gsz) * BM, n0 = (in_group / gsz) * BN;
     const int64_t M = t.M, N = t.N;
     const int tri = t.tri;
     if ((tri == 1 && m0 + BM - 1 < n0) || (tri == 2 && n0 + BN - 1 < m0)) return;
@@ -276,6 +284,12 @@ int tma_bn() { return BN; }
 
 cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st) {
     if (b.n <= 0) return cudaSuccess;
+    static int group_m = -1;
+    if (group_m < 0) {
+        const char *e = getenv("XK_GROUP_M");
+        group_m = (e && *e) ? atoi(e) : 16;
+    }
+    b.group_m = group_m;
     constexpr size_t smem = STAGES * STAGE_BYTES + STAGES * 8 + STAGES * 4 + 1024;
     int total = 0;
     for (int q = 0; q < b.n; ++q) {

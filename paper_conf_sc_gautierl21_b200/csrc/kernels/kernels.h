@@ -37,6 +37,7 @@ struct TmaTask {
 constexpr int kMaxTmaBatch = 16;
 struct TmaBatch {
     int n = 0;
+    int group_m = 16;  // CTA raster: m-blocks per group (L2 reuse); 0 = column-major raster
     int cta_start[kMaxTmaBatch + 1] = {};
     TmaTask t[kMaxTmaBatch];
 };
