@@ -402,6 +402,28 @@ int Runtime::issue(const Rec &R) {
         Buffer *O = buf(R.key, g, true, &rc);
         if (!O) return rc;
         const int64_t idO = (int64_t)R.key * XK_MAX_GPUS + g;
+        if (R.op == XK_OP_TRSM_DIAG || R.op == XK_OP_TRMM_DIAG) {
+            // diagonal solves/multiplies of one step share the diagonal tile of A: grouped
+            // into one recursion over all their B tiles (grouped GEMMs, one base launch)
+            if (!buf(R.keyA, g, false, &rc)) return rc;
+            const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g;
+            PendingBatch &bt = batch_[g];
+            bool conflict = !bt.recs.empty() &&
+                            (bt.op != R.op || bt.recs[0].keyA != R.keyA || bt.recs[0].alpha != R.alpha ||
+                             bt.recs[0].side != R.side || bt.recs[0].uplo != R.uplo || bt.recs[0].ta != R.ta ||
+                             bt.recs[0].diag != R.diag ||
+                             (R.side == 'L' ? bt.recs[0].m != R.m : bt.recs[0].n != R.n));
+            conflict = conflict || (int)bt.recs.size() >= max_batch_ || bt.touches(idO, true) ||
+                       bt.touches(idA, false);
+            for (int q = 0; q < 4 && !conflict; ++q)
+                if (r.dep[q] >= 0 && bt.contains_seq(r.dep[q])) conflict = true;
+            if (conflict && (rc = flush_batch(g))) return rc;
+            bt.recs.push_back(R);
+            bt.out_ids.push_back(idO);
+            bt.in_ids.push_back(idA);
+            bt.op = R.op;
+            return XK_OK;
+        }
         if (R.op != XK_OP_GEMM && R.op != XK_OP_GEMM_TRI) {
             // scale / diagonal-tile ops are launched directly, after this GPU's pending batch
             if ((rc = flush_batch(g))) return rc;
@@ -467,6 +489,7 @@ int Runtime::issue(const Rec &R) {
         const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g, idB = (int64_t)R.keyB * XK_MAX_GPUS + g;
         PendingBatch &bt = batch_[g];
         bool conflict = (int)bt.recs.size() >= max_batch_ ||
+                        (!bt.recs.empty() && (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG)) ||
                         (!bt.recs.empty() && (bt.ta != R.ta || bt.tb != R.tb)) ||
                         bt.touches(idO, true) || bt.touches(idA, false) || bt.touches(idB, false);
         for (int q = 0; q < 4 && !conflict; ++q)
@@ -478,6 +501,7 @@ int Runtime::issue(const Rec &R) {
         bt.in_ids.push_back(idB);
         bt.ta = R.ta;
         bt.tb = R.tb;
+        bt.op = XK_OP_GEMM;
         return XK_OK;
     }
     case XK_REC_D2H: {
@@ -519,6 +543,55 @@ int Runtime::flush_batch(int g) {
     // kernel timing serialises the grouped launches on one stream so that each launch's
     // event-timed duration is its own (no overlap with a concurrent launch)
     cudaStream_t s = kernel_timing ? d.ks[0] : d.ks[batch_count_[g]++ % cfg_.kstreams];
+    if (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG) {
+        const Rec &R0 = bt.recs[0];
+        Buffer *A = buf(R0.keyA, g, false, &rc);
+        if (!A) return rc;
+        double *Bp[kMaxBatch];
+        int64_t ldb[kMaxBatch], other[kMaxBatch];
+        int64_t flops = 0;
+        const int nb = (int)bt.recs.size();
+        for (int q = 0; q < nb; ++q) {
+            const Rec &R = bt.recs[q];
+            for (int j = 0; j < 4; ++j)
+                if ((rc = wait_dep(s, R.r.dep[j]))) return rc;
+            Buffer *O = buf(R.key, g, false, &rc);
+            if (!O) return rc;
+            for (auto &rd : O->readers)
+                if ((rc = wait_on(s, rd))) return rc;
+            if ((rc = wait_on(s, O->writer))) return rc;
+            Bp[q] = O->p;
+            ldb[q] = O->ld;
+            other[q] = (R.side == 'L') ? R.n : R.m;
+            flops += R.r.work;
+        }
+        cudaEvent_t ta = nullptr;
+        if (tracing_ && (rc = trace_begin(g, s, &ta))) return rc;
+        cudaError_t ke = launch_trxm_batch(bt.op == XK_OP_TRSM_DIAG, R0.side, R0.uplo, R0.ta, R0.diag,
+                                           R0.side == 'L' ? R0.m : R0.n, R0.alpha, A->p, A->ld, nb, Bp,
+                                           ldb, other, s);
+        if (ke != cudaSuccess) return cuda_fail(ke, "diagonal-tile kernel launch");
+        if (tracing_)
+            trace_end(g, s, ta, 2, std::string(bt.op == XK_OP_TRSM_DIAG ? "trsm_diag x" : "trmm_diag x") +
+                                       std::to_string(nb), flops);
+        Ev ev;
+        if ((rc = record(s, g, &ev))) return rc;
+        for (int q = 0; q < nb; ++q) {
+            const Rec &R = bt.recs[q];
+            seq_ev_[R.r.seq] = ev;
+            Buffer *O = buf(R.key, g, false, &rc);
+            O->writer = ev;
+            O->readers.clear();
+            stats.tasks[g]++;
+            stats.flops[g] += R.r.work;
+        }
+        add_reader(*A, ev);
+        stats.kernel_launches++;
+        bt.recs.clear();
+        bt.out_ids.clear();
+        bt.in_ids.clear();
+        return XK_OK;
+    }
     TileBatch tb;
     tb.n = (int)bt.recs.size();
     int64_t flops = 0;

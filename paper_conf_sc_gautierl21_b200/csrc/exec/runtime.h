@@ -41,6 +41,7 @@ struct PendingBatch {
     std::vector<Rec> recs;  // copies (records are issued while they are planned)
     std::vector<int64_t> out_ids, in_ids;  // buffer ids written / read
     char ta = 'N', tb = 'N';
+    int op = XK_OP_GEMM;  // GEMM / GEMM_TRI grouped launch, or TRSM_DIAG / TRMM_DIAG sharing keyA
     bool contains_seq(int64_t seq) const {
         for (const Rec &r : recs)
             if (r.r.seq == seq) return true;

@@ -62,6 +62,12 @@ cudaError_t launch_scale_tile(int64_t M, int64_t N, double beta, double *C, int6
 cudaError_t launch_trxm_tile(bool solve, char side, char uplo, char transA, char diag, int64_t M,
                              int64_t N, double alpha, const double *A, int64_t lda, double *B,
                              int64_t ldb, cudaStream_t st);
+// The same on up to kMaxBatch B tiles that share the diagonal tile A (order = the extent
+// along the triangle; other[q] = tile q's extent along the untouched dimension): one
+// recursion whose GEMMs are grouped launches and whose base kernels cover every tile.
+cudaError_t launch_trxm_batch(bool solve, char side, char uplo, char transA, char diag, int64_t order,
+                              double alpha, const double *A, int64_t lda, int n, double *const *B,
+                              const int64_t *ldb, const int64_t *other, cudaStream_t st);
 // S = sym(A) (n x n) from the uplo triangle of A.
 cudaError_t launch_symm_expand(int64_t n, const double *A, int64_t lda, char uplo, double *S,
                                int64_t lds, cudaStream_t st);

@@ -29,35 +29,48 @@ __device__ __forceinline__ double opa(const double *A, int64_t lda, bool trans, 
 //   left  side: v = a column of B (element stride 1, vectors ldb apart), matrix M = op(A)
 //   right side: v = a row of B (element stride ldb, vectors 1 apart),   matrix M = op(A)^T
 // LOWER: M is lower triangular (forward substitution / bottom-up product).
-template <bool SOLVE, bool LOWER>
-__global__ void __launch_bounds__(NB) trxm_base_kernel(int n, int64_t nvec, double alpha,
-                                                       const double *A, int64_t lda, bool mtrans,
-                                                       bool unit, double *B, int64_t es,
-                                                       int64_t vs) {
+// One launch covers the vectors of every B tile of a batch (all share the triangle).
+struct BaseBatch {
+    int n;                            // tiles
+    int cta_start[kMaxBatch + 1];     // CTAs per tile: ceil(nvec / NB)
+    double *B[kMaxBatch];
+    int64_t ldb[kMaxBatch], nvec[kMaxBatch];
+};
+
+template <bool SOLVE, bool LOWER, bool LEFT>
+__global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ BaseBatch bb, int n,
+                                                       double alpha, const double *A, int64_t lda,
+                                                       bool mtrans, bool unit) {
     extern __shared__ double sm[];
     double(*Ms)[NB + 1] = reinterpret_cast<double(*)[NB + 1]>(sm);
     double(*V)[NB + 1] = reinterpret_cast<double(*)[NB + 1]>(sm + NB * (NB + 1));  // V[element][vector]
+    int q = 0;
+#pragma unroll 1
+    while (q + 1 < bb.n && (int)blockIdx.x >= bb.cta_start[q + 1]) ++q;
+    double *B = bb.B[q];
+    const int64_t ldb = bb.ldb[q], nvec = bb.nvec[q];
+    const int64_t es = LEFT ? 1 : ldb, vs = LEFT ? ldb : 1;
     const int tid = threadIdx.x;
-    const int64_t v0 = (int64_t)blockIdx.x * NB;
+    const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * NB;
     // triangle of M into shared memory (only the referenced part is read)
-    for (int q = tid; q < n * n; q += NB) {
-        int r = q % n, c = q / n;
-        bool in = LOWER ? (r > c) : (r < c);
+    for (int r = tid; r < n * n; r += NB) {
+        int i = r % n, c = r / n;
+        bool in = LOWER ? (i > c) : (i < c);
         double x = 0.0;
-        if (in) x = opa(A, lda, mtrans, r, c);
-        else if (r == c) x = unit ? 1.0 : opa(A, lda, mtrans, r, c);
-        Ms[r][c] = x;
+        if (in) x = opa(A, lda, mtrans, i, c);
+        else if (i == c) x = unit ? 1.0 : opa(A, lda, mtrans, i, c);
+        Ms[i][c] = x;
     }
     // vectors of this CTA (coalesced along the contiguous direction)
     const int nv = (int)((nvec - v0) < NB ? (nvec - v0) : NB);
-    if (es == 1) {
-        for (int q = tid; q < n * nv; q += NB) {
-            int e = q % n, v = q / n;
+    if (LEFT) {
+        for (int r = tid; r < n * nv; r += NB) {
+            int e = r % n, v = r / n;
             V[e][v] = B[e + (v0 + v) * vs];
         }
     } else {
-        for (int q = tid; q < n * nv; q += NB) {
-            int v = q % nv, e = q / nv;
+        for (int r = tid; r < n * nv; r += NB) {
+            int v = r % nv, e = r / nv;
             V[e][v] = B[(v0 + v) * vs + e * es];
         }
     }
@@ -95,14 +108,14 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(int n, int64_t nvec, doub
         }
     }
     __syncthreads();
-    if (es == 1) {
-        for (int q = tid; q < n * nv; q += NB) {
-            int e = q % n, v = q / n;
+    if (LEFT) {
+        for (int r = tid; r < n * nv; r += NB) {
+            int e = r % n, v = r / n;
             B[e + (v0 + v) * vs] = V[e][v];
         }
     } else {
-        for (int q = tid; q < n * nv; q += NB) {
-            int v = q % nv, e = q / nv;
+        for (int r = tid; r < n * nv; r += NB) {
+            int v = r % nv, e = r / nv;
             B[(v0 + v) * vs + e * es] = V[e][v];
         }
     }
@@ -112,6 +125,14 @@ struct TriOp {
     bool solve, left, elow, trans, unit;
 };
 
+// The B tiles of one diagonal op: all share the triangle (order n along the triangular
+// dimension); `other` is each tile's extent along the untouched dimension.
+struct Tiles {
+    int n = 0;
+    double *B[kMaxBatch];
+    int64_t ldb[kMaxBatch], other[kMaxBatch];
+};
+
 // op(A) block (rows R0.., cols C0..) as a GEMM operand: pointer + transposition
 inline const double *opa_block(const double *A, int64_t lda, bool trans, int64_t r0, int64_t c0,
                                bool *t) {
@@ -119,104 +140,112 @@ inline const double *opa_block(const double *A, int64_t lda, bool trans, int64_t
     return trans ? A + c0 + r0 * lda : A + r0 + c0 * lda;
 }
 
-cudaError_t base(const TriOp &o, int64_t M, int64_t N, double alpha, const double *A, int64_t lda,
-                 double *B, int64_t ldb, cudaStream_t st) {
-    const int n = (int)(o.left ? M : N);
-    const int64_t nvec = o.left ? N : M;
-    const int64_t es = o.left ? 1 : ldb, vs = o.left ? ldb : 1;
-    // right side: the matrix acting on row vectors is op(A)^T
-    const bool mtrans = o.left ? o.trans : !o.trans;
-    const bool mlow = o.left ? o.elow : !o.elow;
-    const unsigned grid = (unsigned)((nvec + NB - 1) / NB);
+template <bool SOLVE, bool LOWER, bool LEFT>
+cudaError_t base_launch(const BaseBatch &bb, unsigned grid, int n, double alpha, const double *A,
+                        int64_t lda, bool mtrans, bool unit, cudaStream_t st) {
     constexpr size_t smem = 2 * NB * (NB + 1) * sizeof(double);
-    static unsigned attr_set = 0;  // one bit per device
+    auto kern = trxm_base_kernel<SOLVE, LOWER, LEFT>;
+    static unsigned attr_set = 0;  // per instantiation, one bit per device
     int dev = 0;
     cudaGetDevice(&dev);
     if (!(attr_set & (1u << dev))) {
-        cudaError_t e;
-        if ((e = cudaFuncSetAttribute(trxm_base_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-        if ((e = cudaFuncSetAttribute(trxm_base_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-        if ((e = cudaFuncSetAttribute(trxm_base_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-        if ((e = cudaFuncSetAttribute(trxm_base_kernel<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
         attr_set |= 1u << dev;
     }
-    if (o.solve) {
-        if (mlow) trxm_base_kernel<true, true><<<grid, NB, smem, st>>>(n, nvec, alpha, A, lda, mtrans, o.unit, B, es, vs);
-        else trxm_base_kernel<true, false><<<grid, NB, smem, st>>>(n, nvec, alpha, A, lda, mtrans, o.unit, B, es, vs);
-    } else {
-        if (mlow) trxm_base_kernel<false, true><<<grid, NB, smem, st>>>(n, nvec, alpha, A, lda, mtrans, o.unit, B, es, vs);
-        else trxm_base_kernel<false, false><<<grid, NB, smem, st>>>(n, nvec, alpha, A, lda, mtrans, o.unit, B, es, vs);
-    }
+    kern<<<grid, NB, smem, st>>>(bb, n, alpha, A, lda, mtrans, unit);
     return cudaGetLastError();
 }
 
-cudaError_t rec(const TriOp &o, int64_t M, int64_t N, double alpha, const double *A, int64_t lda,
-                double *B, int64_t ldb, cudaStream_t st) {
-    const int64_t n = o.left ? M : N;
-    if (n <= NB) return base(o, M, N, alpha, A, lda, B, ldb, st);
+cudaError_t base(const TriOp &o, int64_t n, const Tiles &T, double alpha, const double *A, int64_t lda,
+                 cudaStream_t st) {
+    BaseBatch bb;
+    bb.n = T.n;
+    int total = 0;
+    for (int q = 0; q < T.n; ++q) {
+        bb.cta_start[q] = total;
+        bb.B[q] = T.B[q];
+        bb.ldb[q] = T.ldb[q];
+        bb.nvec[q] = T.other[q];
+        total += (int)((T.other[q] + NB - 1) / NB);
+    }
+    bb.cta_start[T.n] = total;
+    if (total == 0) return cudaSuccess;
+    // right side: the matrix acting on row vectors is op(A)^T
+    const bool mtrans = o.left ? o.trans : !o.trans;
+    const bool mlow = o.left ? o.elow : !o.elow;
+    const int ni = (int)n;
+#define XK_BASE(S, L, LE) return base_launch<S, L, LE>(bb, (unsigned)total, ni, alpha, A, lda, mtrans, o.unit, st)
+    if (o.solve) {
+        if (mlow) { if (o.left) XK_BASE(true, true, true); else XK_BASE(true, true, false); }
+        else { if (o.left) XK_BASE(true, false, true); else XK_BASE(true, false, false); }
+    } else {
+        if (mlow) { if (o.left) XK_BASE(false, true, true); else XK_BASE(false, true, false); }
+        else { if (o.left) XK_BASE(false, false, true); else XK_BASE(false, false, false); }
+    }
+#undef XK_BASE
+}
+
+// Sub-tiles of every tile: the first n1 (half 1) or the rest (half 2) along the triangle.
+Tiles half(const Tiles &T, bool left, int64_t off) {
+    Tiles H = T;
+    for (int q = 0; q < T.n; ++q) H.B[q] = left ? T.B[q] + off : T.B[q] + off * T.ldb[q];
+    return H;
+}
+
+// One grouped GEMM over the tiles: left  Y = a*opA(blk)*X + b*Y  (Y, X sub-tiles)
+//                                   right Y = a*X*opA(blk) + b*Y
+cudaError_t gemm_all(const TriOp &o, const Tiles &X, const Tiles &Y, const double *P, bool t, int64_t lda,
+                     int64_t ny, int64_t nk, double a, double b, cudaStream_t st) {
+    TileBatch tb;
+    tb.n = X.n;
+    for (int q = 0; q < X.n; ++q) {
+        if (o.left)
+            tb.t[q] = TileTask{P, X.B[q], Y.B[q], lda, X.ldb[q], Y.ldb[q], ny, X.other[q], nk, a, b, 0};
+        else
+            tb.t[q] = TileTask{X.B[q], P, Y.B[q], X.ldb[q], lda, Y.ldb[q], X.other[q], ny, nk, a, b, 0};
+    }
+    return o.left ? launch_dgemm_batch(t, false, tb, st) : launch_dgemm_batch(false, t, tb, st);
+}
+
+cudaError_t rec(const TriOp &o, int64_t n, const Tiles &T, double alpha, const double *A, int64_t lda,
+                cudaStream_t st) {
+    if (n <= NB) return base(o, n, T, alpha, A, lda, st);
     const int64_t n1 = ((n / 2 + NB - 1) / NB) * NB, n2 = n - n1;
     const double *A11 = A, *A22 = A + n1 + n1 * lda;
-    // B halves along the triangular dimension
-    double *B1 = B, *B2 = o.left ? B + n1 : B + n1 * ldb;
-    const int64_t M1 = o.left ? n1 : M, M2 = o.left ? n2 : M;
-    const int64_t N1 = o.left ? N : n1, N2 = o.left ? N : n2;
+    const Tiles B1 = half(T, o.left, 0), B2 = half(T, o.left, n1);
     bool t;
     cudaError_t e;
-    // For the solve the first block solved is the one op(A) maps without coupling:
-    //   left & elow, right & upper: block 1 first; otherwise block 2 first.
-    const bool first1 = (o.left == o.elow);
+    // blocks of op(A): (1,2) = rows 0..n1, cols n1..; (2,1) = rows n1.., cols 0..n1
+    const double *P21 = opa_block(A, lda, o.trans, n1, 0, &t);
+    const double *P12 = opa_block(A, lda, o.trans, 0, n1, &t);
+    // left: Y = op(A)_yx X ; right: Y = X op(A)_xy.  Coupling block for "1 then 2" is
+    // (2,1) on the left and (1,2) on the right, and the reverse for "2 then 1".
     if (o.solve) {
-        if (first1) {
-            if ((e = rec(o, M1, N1, alpha, A11, lda, B1, ldb, st))) return e;
-            if (o.left) {  // B2 = -op(A)21 X1 + alpha B2
-                const double *P = opa_block(A, lda, o.trans, n1, 0, &t);
-                e = launch_dgemm_tile(t, false, n2, N, n1, -1.0, P, lda, B1, ldb, alpha, B2, ldb, st);
-            } else {       // B2 = -X1 op(A)12 + alpha B2
-                const double *P = opa_block(A, lda, o.trans, 0, n1, &t);
-                e = launch_dgemm_tile(false, t, M, n2, n1, -1.0, B1, ldb, P, lda, alpha, B2, ldb, st);
-            }
-            if (e) return e;
-            return rec(o, M2, N2, 1.0, A22, lda, B2, ldb, st);
+        // solve first the block op(A) maps without coupling:
+        //   left & elow, right & upper: block 1 first; otherwise block 2 first.
+        if (o.left == o.elow) {
+            if ((e = rec(o, n1, B1, alpha, A11, lda, st))) return e;
+            if ((e = gemm_all(o, B1, B2, o.left ? P21 : P12, t, lda, n2, n1, -1.0, alpha, st))) return e;
+            return rec(o, n2, B2, 1.0, A22, lda, st);
         }
-        if ((e = rec(o, M2, N2, alpha, A22, lda, B2, ldb, st))) return e;
-        if (o.left) {      // B1 = -op(A)12 X2 + alpha B1
-            const double *P = opa_block(A, lda, o.trans, 0, n1, &t);
-            e = launch_dgemm_tile(t, false, n1, N, n2, -1.0, P, lda, B2, ldb, alpha, B1, ldb, st);
-        } else {           // B1 = -X2 op(A)21 + alpha B1
-            const double *P = opa_block(A, lda, o.trans, n1, 0, &t);
-            e = launch_dgemm_tile(false, t, M, n1, n2, -1.0, B2, ldb, P, lda, alpha, B1, ldb, st);
-        }
-        if (e) return e;
-        return rec(o, M1, N1, 1.0, A11, lda, B1, ldb, st);
+        if ((e = rec(o, n2, B2, alpha, A22, lda, st))) return e;
+        if ((e = gemm_all(o, B2, B1, o.left ? P12 : P21, t, lda, n1, n2, -1.0, alpha, st))) return e;
+        return rec(o, n1, B1, 1.0, A11, lda, st);
     }
     // TRMM (in place): update the block whose inputs must stay old last
     //   left & elow : B2 <- a A22 B2 ; B2 += a A21 B1 ; B1 <- a A11 B1
     //   left & eup  : B1 <- a A11 B1 ; B1 += a A12 B2 ; B2 <- a A22 B2
     //   right & elow: B1 <- a B1 A11 ; B1 += a B2 A21 ; B2 <- a B2 A22
     //   right & eup : B2 <- a B2 A22 ; B2 += a B1 A12 ; B1 <- a B1 A11
-    const bool two_first = (o.left == o.elow);
-    if (two_first) {
-        if ((e = rec(o, M2, N2, alpha, A22, lda, B2, ldb, st))) return e;
-        if (o.left) {
-            const double *P = opa_block(A, lda, o.trans, n1, 0, &t);
-            e = launch_dgemm_tile(t, false, n2, N, n1, alpha, P, lda, B1, ldb, 1.0, B2, ldb, st);
-        } else {
-            const double *P = opa_block(A, lda, o.trans, 0, n1, &t);
-            e = launch_dgemm_tile(false, t, M, n2, n1, alpha, B1, ldb, P, lda, 1.0, B2, ldb, st);
-        }
-        if (e) return e;
-        return rec(o, M1, N1, alpha, A11, lda, B1, ldb, st);
+    if (o.left == o.elow) {
+        if ((e = rec(o, n2, B2, alpha, A22, lda, st))) return e;
+        if ((e = gemm_all(o, B1, B2, o.left ? P21 : P12, t, lda, n2, n1, alpha, 1.0, st))) return e;
+        return rec(o, n1, B1, alpha, A11, lda, st);
     }
-    if ((e = rec(o, M1, N1, alpha, A11, lda, B1, ldb, st))) return e;
-    if (o.left) {
-        const double *P = opa_block(A, lda, o.trans, 0, n1, &t);
-        e = launch_dgemm_tile(t, false, n1, N, n2, alpha, P, lda, B2, ldb, 1.0, B1, ldb, st);
-    } else {
-        const double *P = opa_block(A, lda, o.trans, n1, 0, &t);
-        e = launch_dgemm_tile(false, t, M, n1, n2, alpha, B2, ldb, P, lda, 1.0, B1, ldb, st);
-    }
-    if (e) return e;
-    return rec(o, M2, N2, alpha, A22, lda, B2, ldb, st);
+    if ((e = rec(o, n1, B1, alpha, A11, lda, st))) return e;
+    if ((e = gemm_all(o, B2, B1, o.left ? P12 : P21, t, lda, n1, n2, alpha, 1.0, st))) return e;
+    return rec(o, n2, B2, alpha, A22, lda, st);
 }
 
 __global__ void symm_expand_kernel(int64_t n, const double *A, int64_t lda, bool lower, double *S,
@@ -242,17 +271,42 @@ __global__ void scale_tri_kernel(int64_t M, int64_t N, double beta, double *C, i
 
 }  // namespace
 
-cudaError_t launch_trxm_tile(bool solve, char side, char uplo, char transA, char diag, int64_t M,
-                             int64_t N, double alpha, const double *A, int64_t lda, double *B,
-                             int64_t ldb, cudaStream_t st) {
-    if (M <= 0 || N <= 0) return cudaSuccess;
+static TriOp make_op(bool solve, char side, char uplo, char transA, char diag) {
     TriOp o;
     o.solve = solve;
     o.left = (side == 'L' || side == 'l');
     o.trans = (transA == 'T' || transA == 't' || transA == 'C' || transA == 'c');
     o.elow = ((uplo == 'L' || uplo == 'l') != o.trans);
     o.unit = (diag == 'U' || diag == 'u');
-    return rec(o, M, N, alpha, A, lda, B, ldb, st);
+    return o;
+}
+
+cudaError_t launch_trxm_tile(bool solve, char side, char uplo, char transA, char diag, int64_t M,
+                             int64_t N, double alpha, const double *A, int64_t lda, double *B,
+                             int64_t ldb, cudaStream_t st) {
+    if (M <= 0 || N <= 0) return cudaSuccess;
+    TriOp o = make_op(solve, side, uplo, transA, diag);
+    Tiles T;
+    T.n = 1;
+    T.B[0] = B;
+    T.ldb[0] = ldb;
+    T.other[0] = o.left ? N : M;
+    return rec(o, o.left ? M : N, T, alpha, A, lda, st);
+}
+
+cudaError_t launch_trxm_batch(bool solve, char side, char uplo, char transA, char diag, int64_t order,
+                              double alpha, const double *A, int64_t lda, int n, double *const *B,
+                              const int64_t *ldb, const int64_t *other, cudaStream_t st) {
+    if (order <= 0 || n <= 0) return cudaSuccess;
+    TriOp o = make_op(solve, side, uplo, transA, diag);
+    Tiles T;
+    T.n = n;
+    for (int q = 0; q < n; ++q) {
+        T.B[q] = B[q];
+        T.ldb[q] = ldb[q];
+        T.other[q] = other[q];
+    }
+    return rec(o, order, T, alpha, A, lda, st);
 }
 
 cudaError_t launch_symm_expand(int64_t n, const double *A, int64_t lda, char uplo, double *S,
