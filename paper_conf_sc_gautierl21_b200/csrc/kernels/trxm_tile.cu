@@ -74,38 +74,64 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ B
             V[e][v] = B[(v0 + v) * vs + e * es];
         }
     }
+    // pad the triangle to NB with the identity and the vectors with zeros, so the fully
+    // unrolled register code below always works on NB x NB (padded rows stay zero and are
+    // never stored)
+    for (int r = tid; r < NB * NB; r += NB) {
+        int i = r % NB, c = r / NB;
+        if (i >= n || c >= n) Ms[i][c] = (i == c) ? 1.0 : 0.0;
+    }
+    for (int r = tid; r < NB * NB; r += NB) {
+        int e = r % NB, v = r / NB;
+        if (e >= n || v >= nv) V[e][v] = 0.0;
+    }
     __syncthreads();
-    if (tid < nv) {
+    {
+        // one vector per thread, held in registers; every loop is fully unrolled so the
+        // indices are compile-time and independent updates interleave (ILP)
         const int v = tid;
+        double x[NB];
+#pragma unroll
+        for (int i = 0; i < NB; ++i) x[i] = V[i][v];
         if (SOLVE) {
-            if (LOWER) {
-                for (int i = 0; i < n; ++i) {
-                    double s = alpha * V[i][v];
-                    for (int l = 0; l < i; ++l) s -= Ms[i][l] * V[l][v];
-                    V[i][v] = unit ? s : s / Ms[i][i];
+#pragma unroll
+            for (int i = 0; i < NB; ++i) x[i] *= alpha;
+            if (LOWER) {  // column-oriented forward substitution: x_i -= M_il x_l, l ascending
+#pragma unroll
+                for (int l = 0; l < NB; ++l) {
+                    if (!unit) x[l] = x[l] / Ms[l][l];
+#pragma unroll
+                    for (int i = l + 1; i < NB; ++i) x[i] -= Ms[i][l] * x[l];
                 }
-            } else {
-                for (int i = n - 1; i >= 0; --i) {
-                    double s = alpha * V[i][v];
-                    for (int l = i + 1; l < n; ++l) s -= Ms[i][l] * V[l][v];
-                    V[i][v] = unit ? s : s / Ms[i][i];
+            } else {      // back substitution, l descending
+#pragma unroll
+                for (int l = NB - 1; l >= 0; --l) {
+                    if (!unit) x[l] = x[l] / Ms[l][l];
+#pragma unroll
+                    for (int i = 0; i < l; ++i) x[i] -= Ms[i][l] * x[l];
                 }
             }
         } else {
-            if (LOWER) {  // bottom-up keeps the inputs of later rows intact
-                for (int i = n - 1; i >= 0; --i) {
+            if (LOWER) {  // bottom-up: row i only reads x_0..x_i, still unmodified
+#pragma unroll
+                for (int i = NB - 1; i >= 0; --i) {
                     double s = 0.0;
-                    for (int l = 0; l <= i; ++l) s += Ms[i][l] * V[l][v];
-                    V[i][v] = alpha * s;
+#pragma unroll
+                    for (int l = 0; l <= i; ++l) s += Ms[i][l] * x[l];
+                    x[i] = alpha * s;
                 }
             } else {
-                for (int i = 0; i < n; ++i) {
+#pragma unroll
+                for (int i = 0; i < NB; ++i) {
                     double s = 0.0;
-                    for (int l = i; l < n; ++l) s += Ms[i][l] * V[l][v];
-                    V[i][v] = alpha * s;
+#pragma unroll
+                    for (int l = i; l < NB; ++l) s += Ms[i][l] * x[l];
+                    x[i] = alpha * s;
                 }
             }
         }
+#pragma unroll
+        for (int i = 0; i < NB; ++i) V[i][v] = x[i];
     }
     __syncthreads();
     if (LEFT) {
