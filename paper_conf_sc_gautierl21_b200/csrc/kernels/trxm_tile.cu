@@ -52,7 +52,9 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ B
     const int64_t es = LEFT ? 1 : ldb, vs = LEFT ? ldb : 1;
     const int tid = threadIdx.x;
     const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * NB;
-    // triangle of M into shared memory (only the referenced part is read)
+    // triangle of M into shared memory (only the referenced part is read); the load loops
+    // are unrolled so many global loads are in flight per thread (the kernel is latency-bound)
+#pragma unroll 16
     for (int r = tid; r < n * n; r += NB) {
         int i = r % n, c = r / n;
         bool in = LOWER ? (i > c) : (i < c);
@@ -64,11 +66,13 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ B
     // vectors of this CTA (coalesced along the contiguous direction)
     const int nv = (int)((nvec - v0) < NB ? (nvec - v0) : NB);
     if (LEFT) {
+#pragma unroll 16
         for (int r = tid; r < n * nv; r += NB) {
             int e = r % n, v = r / n;
             V[e][v] = B[e + (v0 + v) * vs];
         }
     } else {
+#pragma unroll 16
         for (int r = tid; r < n * nv; r += NB) {
             int v = r % nv, e = r / nv;
             V[e][v] = B[(v0 + v) * vs + e * es];
@@ -135,11 +139,13 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ B
     }
     __syncthreads();
     if (LEFT) {
+#pragma unroll 16
         for (int r = tid; r < n * nv; r += NB) {
             int e = r % n, v = r / n;
             B[e + (v0 + v) * vs] = V[e][v];
         }
     } else {
+#pragma unroll 16
         for (int r = tid; r < n * nv; r += NB) {
             int v = r % nv, e = r / nv;
             B[(v0 + v) * vs + e * es] = V[e][v];
