@@ -93,6 +93,7 @@ int Runtime::init(const xk_config_t &cfg) {
     ev_used_.assign(G, {});
     batch_.assign(G, PendingBatch());
     batch_count_.assign(G, 0);
+    batches_in_call_.assign(G, 0);
     {
         const char *eb = std::getenv("XK_BATCH");
         int mb = (eb && *eb) ? std::atoi(eb) : 16;
@@ -488,7 +489,11 @@ int Runtime::issue(const Rec &R) {
         if (!buf(R.keyA, g, false, &rc) || !buf(R.keyB, g, false, &rc)) return rc;
         const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g, idB = (int64_t)R.keyB * XK_MAX_GPUS + g;
         PendingBatch &bt = batch_[g];
-        bool conflict = (int)bt.recs.size() >= max_batch_ ||
+        // batch size ramps 1, 2, 4, ... up to max_batch_ at the start of each call, so the
+        // first kernels start as soon as their own inputs have landed instead of waiting
+        // for a whole batch worth of tiles to cross PCIe
+        const int cap = (int)std::min<int64_t>(max_batch_, (int64_t)1 << std::min<int64_t>(batches_in_call_[g], 5));
+        bool conflict = (int)bt.recs.size() >= cap ||
                         (!bt.recs.empty() && (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG)) ||
                         (!bt.recs.empty() && (bt.ta != R.ta || bt.tb != R.tb)) ||
                         bt.touches(idO, true) || bt.touches(idA, false) || bt.touches(idB, false);
@@ -639,6 +644,7 @@ int Runtime::flush_batch(int g) {
         stats.flops[g] += R.r.work;
     }
     stats.kernel_launches++;
+    batches_in_call_[g]++;
     bt.recs.clear();
     bt.out_ids.clear();
     bt.in_ids.clear();
@@ -982,6 +988,7 @@ int Runtime::run(const xk_call_t &call, bool wait) {
     std::vector<Rec> recs;
     std::string err;
     size_t d2h0 = pending_d2h_.size();
+    std::fill(batches_in_call_.begin(), batches_in_call_.end(), 0);
     // records are issued as the planner produces them: the GPUs start on the first copies
     // and tasks while the rest of the call is still being planned
     Planner::Sink sink = [this](const Rec &r) { return issue(r); };

@@ -143,6 +143,7 @@ private:
     int cur_dev_ = -1;
     std::vector<PendingBatch> batch_;
     std::vector<int64_t> batch_count_;
+    std::vector<int64_t> batches_in_call_;  // grouped launches issued in the current call, per GPU
     int max_batch_ = kMaxBatch;
     int nks_ = 4;  // kernel streams created per GPU
 };
