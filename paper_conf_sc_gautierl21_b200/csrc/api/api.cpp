@@ -140,7 +140,7 @@ int xk_finalize(void) {
 
 int xk_register(void *p, size_t bytes) {
     if (!runtime()) return need_init();
-    return runtime()->register_host(p, bytes, false);
+    return runtime()->register_host(p, bytes);
 }
 
 int xk_unregister(void *p) {

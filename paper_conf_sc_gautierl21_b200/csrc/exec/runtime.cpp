@@ -428,8 +428,7 @@ int Runtime::issue(const Rec &R) {
         if (R.op != XK_OP_GEMM && R.op != XK_OP_GEMM_TRI) {
             // scale / diagonal-tile ops are launched directly, after this GPU's pending batch
             if ((rc = flush_batch(g))) return rc;
-            // independent diagonal-tile ops of one step (e.g. the TRSM solves of every column
-            // of tiles) spread over all kernel streams so they overlap
+            // independent scale / SYMM-diagonal ops spread over all kernel streams
             const uint64_t h = (uint64_t)(e.bi * 7919 + e.bj * 104729);
             cudaStream_t s = devs_[g].ks[h % (uint64_t)nks_];
             for (int q = 0; q < 4; ++q)
@@ -446,9 +445,6 @@ int Runtime::issue(const Rec &R) {
             if (tracing_ && (rc = trace_begin(g, s, &ta))) return rc;
             if (R.op == XK_OP_SCALE) {
                 ke = launch_scale_tri(R.m, R.n, R.beta, O->p, O->ld, R.tri, s);
-            } else if (R.op == XK_OP_TRSM_DIAG || R.op == XK_OP_TRMM_DIAG) {
-                ke = launch_trxm_tile(R.op == XK_OP_TRSM_DIAG, R.side, R.uplo, R.ta, R.diag, R.m, R.n,
-                                      R.alpha, A->p, A->ld, O->p, O->ld, s);
             } else if (R.op == XK_OP_SYMM_DIAG) {
                 // expand the diagonal tile of A symmetrically into a scratch tile, then GEMM
                 const int64_t ka = (R.side == 'L') ? R.m : R.n;
@@ -865,9 +861,8 @@ void Runtime::release_internal_pins() {
     internal_reg_.clear();
 }
 
-int Runtime::register_host(void *p, size_t bytes, bool internal) {
+int Runtime::register_host(void *p, size_t bytes) {
     std::lock_guard<std::recursive_mutex> lk(mu);
-    (void)internal;
     if (!p || bytes == 0) return XK_OK;
     cudaError_t e = cudaHostRegister(p, bytes, cudaHostRegisterPortable);
     if (e == cudaErrorHostMemoryAlreadyRegistered) {
@@ -944,7 +939,19 @@ int Runtime::sync_all() {
 
 int Runtime::run(const xk_call_t &call, bool wait) {
     std::lock_guard<std::recursive_mutex> lk(mu);
+    if (failed_) {
+        set_error("an earlier CUDA failure left the tile cache inconsistent: xk_finalize() and xk_init() again");
+        return failed_;
+    }
     cur_dev_ = -1;
+    int rc = run_impl(call, wait);
+    // after a runtime failure mid-call the directory may describe copies that were never
+    // made: refuse further work until re-initialisation (never compute on a stale cache)
+    if (rc == XK_ERR_CUDA || rc == XK_ERR_OOM || rc == XK_ERR_INTERNAL) failed_ = rc;
+    return rc;
+}
+
+int Runtime::run_impl(const xk_call_t &call, bool wait) {
     int rc;
     // page-lock the operands the call touches (excluded from timings when the caller
     // registered them first with xk_register)

@@ -80,7 +80,7 @@ public:
     int sync_all();
     int invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld);
 
-    int register_host(void *p, size_t bytes, bool internal);
+    int register_host(void *p, size_t bytes);
     int unregister_host(void *p);
     int ensure_pinned(uint64_t base, int64_t rows, int64_t cols, int64_t ld);
 
@@ -94,6 +94,8 @@ public:
     std::recursive_mutex mu;
 
 private:
+    int run_impl(const xk_call_t &call, bool wait);
+    int failed_ = 0;  // sticky runtime failure (XK_ERR_*), cleared by re-initialisation
     int issue(const Rec &r);
     int flush_batch(int g);
     int flush_for(const Rec &r);
