@@ -248,3 +248,29 @@ def test_trace_timeline(tmp_path):
     assert by["P2P-in"] == sum(st["p2p_in_bytes"]) > 0
     assert any(e["tid"] == "kernels" for e in ev)
     assert st["trace_ms"]["kernel"] > 0 and st["trace_ms"]["h2d"] > 0
+
+
+def test_out_of_memory_fails_cleanly():
+    """No eviction: when the device tile cache cannot grow, the call returns
+    XK_ERR_OOM instead of crashing, later calls refuse to run on the inconsistent cache, and
+    re-initialisation recovers."""
+    import torch
+    N, T = 8192, 2048
+    A, B, C = inputs.uniform(1, N, N), inputs.uniform(2, N, N), inputs.uniform(3, N, N)
+    free, _ = torch.cuda.mem_get_info()
+    hog = torch.empty(int(free - (600 << 20)) // 8, dtype=torch.float64, device="cuda")  # leave ~600 MB
+    try:
+        xk.init(ngpus=1, tile=T, probe=False)
+        with pytest.raises(xk.XKError) as e:
+            xk.dgemm("N", "N", N, N, N, 1.0, A, N, B, N, 0.0, C, N)  # needs 1.5 GB of tiles
+        assert e.value.code == 3  # XK_ERR_OOM
+        with pytest.raises(xk.XKError):
+            xk.dgemm("N", "N", N, N, N, 1.0, A, N, B, N, 0.0, C, N)  # sticky until re-init
+        xk.finalize()
+    finally:
+        del hog
+        torch.cuda.empty_cache()
+    xk.init(ngpus=1, tile=T, probe=False)
+    C2 = np.zeros((N, N), order="F")
+    assert xk.dgemm("N", "N", 512, 512, 512, 1.0, A, N, B, N, 0.0, C2, N) == 0
+    xk.finalize()
