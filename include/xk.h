@@ -174,6 +174,8 @@ typedef struct xk_stats {
     double kernel_ms_total;          /* summed tile-kernel launch time (when timing on) */
     int64_t kernel_timed_launches;   /* launches included in kernel_ms_total */
     int64_t kernel_timed_flops;      /* algorithmic flops of those launches (2*m*n*k per task) */
+    int64_t link_bytes[(XK_MAX_GPUS + 1) * (XK_MAX_GPUS + 1)]; /* bytes per link, row = source,
+                                        column = destination, stride ngpus+1, index ngpus = host */
     double trace_ms[4];              /* with tracing on: summed op time by kind
                                         [H2D, P2P, kernel, D2H] (paper Fig. 6 breakdown) */
 } xk_stats_t;

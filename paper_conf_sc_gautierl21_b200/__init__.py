@@ -169,6 +169,7 @@ def get_stats():
               "kernel_ms_total", "kernel_timed_launches", "kernel_timed_flops"):
         out[f] = getattr(st, f)
     out["trace_ms"] = dict(zip(("h2d", "p2p", "kernel", "d2h"), list(st.trace_ms)))
+    out["link_bytes"] = [[st.link_bytes[s * (G + 1) + d] for d in range(G + 1)] for s in range(G + 1)]
     return out
 
 

@@ -47,6 +47,7 @@ class Stats(ctypes.Structure):
                 ("forwards_inflight", i64), ("forwards_valid", i64), ("kernel_launches", i64),
                 ("host_registrations", i64), ("kernel_ms_total", c_double),
                 ("kernel_timed_launches", i64), ("kernel_timed_flops", i64),
+                ("link_bytes", i64 * ((MAX_GPUS + 1) * (MAX_GPUS + 1))),
                 ("trace_ms", c_double * 4)]
 
 

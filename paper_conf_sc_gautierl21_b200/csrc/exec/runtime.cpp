@@ -364,6 +364,7 @@ int Runtime::issue(const Rec &R) {
         B->writer = ev;
         B->readers.clear();
         stats.h2d_bytes[g] += r.work;
+        stats.link_bytes[(size_t)devs_.size() * (devs_.size() + 1) + g] += r.work;
         return XK_OK;
     }
     case XK_REC_P2P: {
@@ -393,6 +394,7 @@ int Runtime::issue(const Rec &R) {
         add_reader(*S, ev);
         stats.p2p_in_bytes[g] += r.work;
         stats.p2p_out_bytes[gs] += r.work;
+        stats.link_bytes[(size_t)gs * (devs_.size() + 1) + g] += r.work;
         if (r.src_state == XK_SRC_INFLIGHT) stats.forwards_inflight++;
         else stats.forwards_valid++;
         return XK_OK;
@@ -526,6 +528,7 @@ int Runtime::issue(const Rec &R) {
         add_reader(*S, ev);
         pending_d2h_.push_back(ev);
         stats.d2h_bytes[gs] += r.work;
+        stats.link_bytes[(size_t)gs * (devs_.size() + 1) + devs_.size()] += r.work;
         return XK_OK;
     }
     default:

@@ -111,6 +111,9 @@ def test_heuristic_modes_same_numbers_bytes_follow_plan(mode, opt):
     assert np.array_equal(C, Cref)
     tile_b = 8 * T * T
     h2d, p2p = sum(st["h2d_bytes"]), sum(st["p2p_in_bytes"])
+    L = st["link_bytes"]  # per-link matrix agrees with the per-GPU counters
+    assert sum(L[G][g] for g in range(G)) == h2d and sum(L[g][G] for g in range(G)) == sum(st["d2h_bytes"])
+    assert sum(L[s][d] for s in range(G) for d in range(G)) == p2p
     assert sum(st["d2h_bytes"]) == t * t * tile_b
     rA, rB = 2, 4  # min(Q, t), min(P, t)
     if mode == "home":
