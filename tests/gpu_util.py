@@ -15,3 +15,11 @@ def from_dev(t, ld, ncols):
 def stream_ptr():
     import torch
     return torch.cuda.current_stream().cuda_stream
+
+
+def device_map(G):
+    """Logical GPU -> physical device: distinct devices when the box has at least G of them
+    (real NVLink peer copies), else all on device 0 (logical-device mode)."""
+    import torch
+    n = torch.cuda.device_count()
+    return list(range(G)) if n >= G else [0] * G

@@ -15,6 +15,7 @@ import pytest
 import inputs
 import oracle
 import paper_conf_sc_gautierl21_b200 as xk
+from tests.gpu_util import device_map
 
 pytestmark = pytest.mark.gpu
 EPS = 2.0 ** -53
@@ -31,7 +32,7 @@ def tri_mask(n, lower):
 @pytest.fixture(params=[1, 4], ids=["G1", "G4"])
 def lib(request):
     G = request.param
-    xk.init(ngpus=G, phys=[0] * G, tile=128, probe=False)
+    xk.init(ngpus=G, phys=device_map(G), tile=128, probe=False)
     yield G
     xk.finalize()
 
@@ -160,7 +161,7 @@ def test_trsm_gemm_composition():
     G, T, N = 4, 128, 384
     L = inputs.tri_dd(4, N, lower=True, fill=np.nan)
     B0 = inputs.uniform(2, N, N); D = inputs.uniform(5, N, N)
-    xk.init(ngpus=G, phys=[0] * G, tile=T, probe=False)
+    xk.init(ngpus=G, phys=device_map(G), tile=T, probe=False)
     try:
         Xs = B0.copy(order="F"); Cs = np.zeros((N, N), order="F")
         xk.dtrsm("L", "L", "N", "N", N, N, 1.5, L, N, Xs, N)

@@ -11,6 +11,7 @@ import pytest
 import inputs
 import oracle
 import paper_conf_sc_gautierl21_b200 as xk
+from tests.gpu_util import device_map
 
 pytestmark = pytest.mark.gpu
 
@@ -27,7 +28,7 @@ def lib1():
 
 
 def logical(G, **kw):
-    xk.init(ngpus=G, phys=[0] * G, probe=False, **kw)
+    xk.init(ngpus=G, phys=device_map(G), probe=False, **kw)
 
 
 def check_bound(ta, tb, m, n, k, alpha, A, B, beta, C0, got, ref):

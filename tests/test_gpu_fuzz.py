@@ -9,6 +9,7 @@ import pytest
 import inputs
 import oracle
 import paper_conf_sc_gautierl21_b200 as xk
+from tests.gpu_util import device_map
 
 pytestmark = pytest.mark.gpu
 EPS = 2.0 ** -53
@@ -31,7 +32,7 @@ def test_random_calls(seed):
     r = random.Random(seed)
     G = r.choice([1, 2, 3])
     T = r.choice([64, 96, 128])
-    xk.init(ngpus=G, phys=[0] * G, tile=T, probe=False, topo=r.choice(["ranked", "unranked", "home"]),
+    xk.init(ngpus=G, phys=device_map(G), tile=T, probe=False, topo=r.choice(["ranked", "unranked", "home"]),
             optimistic=r.random() < 0.7)
     try:
         for _ in range(8):
