@@ -1,0 +1,30 @@
+"""Plan-predicted heuristic ablation on 8 GPUs (virtual-time model of the planner; no GPU):
+makespan = max t_end of the plan, for the paper's DGX-1 (Fig. 2 matrix, PCIe Gen3 host links,
+V100 FP64 rate) and an 8x B200 NVSwitch box (measured single-GPU PCIe/NVLink/FP64 rates).
+Informative only: the model's timing fidelity is not pinned."""
+import json, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_sc_gautierl21_b200 as xk
+from tests.test_planner import fig2, with_host, uniform
+
+MODES = [("full", "ranked", True), ("no_opt", "ranked", False), ("no_opt_topo", "unranked", False), ("home", "home", True)]
+boxes = {
+    # DGX-1: Fig. 2 GPU matrix; host links PCIe Gen3 x16 shared by 2 GPUs -> ~6 GB/s each
+    "dgx1_v100": (with_host(fig2(), host=6000), 7000000),
+    # 8x B200: 55 GB/s PCIe Gen5 per GPU (measured), ~700 GB/s CE peer copies, 35 TF tile rate (measured)
+    "hgx_b200": (uniform(8, peer=700000, host=55000), 35000000),
+}
+out = {}
+for box, (bw, rate) in boxes.items():
+    for N in (16384, 32768):
+        T = 2048
+        call = xk.make_call(m=N, n=N, k=N, alpha=1.0, beta=1.0, A=1 << 40, lda=N, B=2 << 40, ldb=N, C=3 << 40, ldc=N, sync=True)
+        row = {}
+        for name, topo, opt in MODES:
+            recs = xk.plan_dump(call, bw, rate_mflops=rate, topo=topo, optimistic=opt, tile=T, cap=1 << 18)
+            t = max(r[12] for r in recs) * 1e-9
+            h2d = sum(r[13] for r in recs if r[1] == 0) / 1e9
+            row[name] = {"pred_tflops": round(2.0 * N ** 3 / t / 1e12, 2), "h2d_GB": round(h2d, 2)}
+        out["%s_N%d" % (box, N)] = row
+        print(box, N, json.dumps(row))
+print(json.dumps(out))
