@@ -68,3 +68,9 @@ def test_product_never_imports_the_oracle():
                 txt = open(os.path.join(dirpath, fn)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, fn
                 assert "oracle.h" not in txt and "liboracle" not in txt, fn
+
+
+def test_c_example_builds_against_the_header():
+    """The C ABI is usable from plain C: examples/xk_dgemm_example.c compiles and links."""
+    from tools.build_native import build_example
+    assert os.path.exists(build_example())

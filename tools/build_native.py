@@ -88,11 +88,23 @@ def build_xk(force=False, verbose=False):
     return out
 
 
+def build_example(force=False):
+    """examples/xk_dgemm_example.c linked against libxk.so (the C ABI used from plain C)."""
+    src = os.path.join(ROOT, "examples", "xk_dgemm_example.c")
+    out = os.path.join(ROOT, "examples", "xk_dgemm_example")
+    lib = build_xk()
+    if force or _stale(out, [src, lib, os.path.join(ROOT, "include", "xk.h")]):
+        _run(["gcc", "-O2", "-Wall", "-I", os.path.join(ROOT, "include"), src, "-L", PKG, "-lxk",
+              "-Wl,-rpath," + PKG, "-lm", "-o", out])
+    return out
+
+
 def build_all(force=False):
     build_inputs(force)
     build_oracle(force)
     if os.path.isdir(os.path.join(PKG, "csrc")):
         build_xk(force)
+        build_example(force)
 
 
 if __name__ == "__main__":
