@@ -208,22 +208,45 @@ def test_full_size_n16384_exact_freivalds():
         assert np.array_equal(lhs, rhs)
 
 
-def test_full_size_n32768_sampled():
-    """The bench workload (N=32768, T=2048, G=1, uniform [-1,1)): 4096 sampled entries vs
-    the oracle's dot loop under the elementwise bound."""
-    N, T = 32768, 2048
-    A, B, C0 = inputs.uniform(1, N, N), inputs.uniform(2, N, N), inputs.uniform(3, N, N)
-    C = C0.copy(order="F")
-    xk.init(ngpus=1, tile=T, probe=False)
-    xk.register(A); xk.register(B); xk.register(C)
-    assert xk.dgemm("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N) == 0
-    xk.finalize()
+@pytest.mark.parametrize("N,T", [(32768, 4096), (32768, 2048), (65536, 4096)])
+def test_full_size_sampled(N, T):
+    """The bench workload (N=32768, T=4096 -- bench.py's launch configuration -- and T=2048)
+    and the largest BASELINE size (N=65536), G=1, uniform [-1,1): 4096 sampled entries vs the
+    oracle's dot loop under the elementwise bound."""
+    A, B, C = inputs.uniform(1, N, N), inputs.uniform(2, N, N), inputs.uniform(3, N, N)
     rng = np.random.default_rng(7)
     ii = rng.integers(0, N, 4096); jj = rng.integers(0, N, 4096)
     ii[:4] = [0, N - 1, 0, N - 1]; jj[:4] = [0, 0, N - 1, N - 1]
-    ref = oracle.dgemm_sampled("N", "N", N, 1.5, A, B, -0.75, C0[ii, jj], ii, jj)
-    mag = 1.5 * np.einsum("qk,kq->q", np.abs(A[ii, :]), np.abs(B[:, jj])) + 0.75 * np.abs(C0[ii, jj])
+    c0 = C[ii, jj].copy()  # C is overwritten in place; keep only the sampled inputs
+    xk.init(ngpus=1, tile=T, probe=False)
+    try:
+        xk.register(A); xk.register(B); xk.register(C)
+        assert xk.dgemm("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N) == 0
+    finally:
+        xk.finalize()
+    ref = oracle.dgemm_sampled("N", "N", N, 1.5, A, B, -0.75, c0, ii, jj)
+    mag = 1.5 * np.einsum("qk,kq->q", np.abs(A[ii, :]), np.abs(B[:, jj])) + 0.75 * np.abs(c0)
     assert np.all(np.abs(C[ii, jj] - ref) <= 4 * N * 2.0 ** -53 * mag)
+
+
+def test_empty_and_degenerate_calls(lib1):
+    """m = 0, n = 0, k = 0 and alpha = 0 cases after init: no work or C <- beta*C only."""
+    A = inputs.uniform(1, 64, 64)
+    C0 = inputs.uniform(3, 64, 64)
+    xk.reset_stats()
+    C = C0.copy(order="F")
+    assert xk.dgemm("N", "N", 0, 64, 64, 1.0, A, 64, A, 64, 0.0, C, 64) == 0
+    assert xk.dgemm("N", "N", 64, 0, 64, 1.0, A, 64, A, 64, 0.0, C, 64) == 0
+    assert xk.get_stats()["tasks"][0] == 0 and np.array_equal(C, C0)
+    assert xk.dgemm("N", "N", 64, 64, 0, 1.0, A, 64, A, 64, -2.0, C, 64) == 0  # k = 0: C <- beta*C
+    assert np.array_equal(C, -2.0 * C0)
+    C = C0.copy(order="F")
+    assert xk.dgemm("N", "N", 64, 64, 64, 0.0, A, 64, A, 64, 0.0, C, 64) == 0  # alpha = beta = 0
+    assert np.all(C == 0)
+    C = C0.copy(order="F")
+    assert xk.dgemm("N", "N", 1, 1, 1, 1.5, A, 64, A, 64, 1.0, C, 64) == 0  # 1 x 1 x 1
+    assert C[0, 0] == C0[0, 0] + 1.5 * A[0, 0] * A[0, 0]
+    assert np.array_equal(C[1:], C0[1:]) and np.array_equal(C[:, 1:], C0[:, 1:])
 
 
 def test_trace_timeline(tmp_path):
