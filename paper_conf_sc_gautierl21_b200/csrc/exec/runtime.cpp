@@ -485,7 +485,9 @@ int Runtime::issue(const Rec &R) {
             return XK_OK;
         }
         if (!buf(R.keyA, g, false, &rc) || !buf(R.keyB, g, false, &rc)) return rc;
+        if (R.keyC2 >= 0 && !buf(R.keyC2, g, false, &rc)) return rc;
         const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g, idB = (int64_t)R.keyB * XK_MAX_GPUS + g;
+        const int64_t idC2 = R.keyC2 >= 0 ? (int64_t)R.keyC2 * XK_MAX_GPUS + g : -1;
         PendingBatch &bt = batch_[g];
         // batch size ramps 1, 2, 4, ... up to max_batch_ at the start of each call, so the
         // first kernels start as soon as their own inputs have landed instead of waiting
@@ -494,7 +496,8 @@ int Runtime::issue(const Rec &R) {
         bool conflict = (int)bt.recs.size() >= cap ||
                         (!bt.recs.empty() && (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG)) ||
                         (!bt.recs.empty() && (bt.ta != R.ta || bt.tb != R.tb)) ||
-                        bt.touches(idO, true) || bt.touches(idA, false) || bt.touches(idB, false);
+                        bt.touches(idO, true) || bt.touches(idA, false) || bt.touches(idB, false) ||
+                        (idC2 >= 0 && bt.touches(idC2, false));
         for (int q = 0; q < 4 && !conflict; ++q)
             if (r.dep[q] >= 0 && bt.contains_seq(r.dep[q])) conflict = true;
         if (conflict && (rc = flush_batch(g))) return rc;
@@ -502,6 +505,7 @@ int Runtime::issue(const Rec &R) {
         bt.out_ids.push_back(idO);
         bt.in_ids.push_back(idA);
         bt.in_ids.push_back(idB);
+        if (idC2 >= 0) bt.in_ids.push_back(idC2);
         bt.ta = R.ta;
         bt.tb = R.tb;
         bt.op = XK_OP_GEMM;
@@ -610,7 +614,10 @@ int Runtime::flush_batch(int g) {
         for (auto &rd : O->readers)
             if ((rc = wait_on(s, rd))) return rc;
         if ((rc = wait_on(s, O->writer))) return rc;
-        tb.t[q] = TileTask{A->p, B->p, O->p, A->ld, B->ld, O->ld, R.m, R.n, R.k, R.alpha, R.beta, R.tri};
+        Buffer *C2 = nullptr;
+        if (R.keyC2 >= 0 && !(C2 = buf(R.keyC2, g, false, &rc))) return rc;
+        tb.t[q] = TileTask{A->p, B->p, O->p, A->ld, B->ld, O->ld, R.m, R.n, R.k, R.alpha, R.beta, R.tri,
+                           C2 ? C2->p : nullptr, C2 ? C2->ld : 0, C2 ? R.beta2 : 0.0};
         flops += R.r.work;
     }
     cudaEvent_t t0 = nullptr, t1 = nullptr;
@@ -639,6 +646,7 @@ int Runtime::flush_batch(int g) {
         O->readers.clear();
         add_reader(*buf(R.keyA, g, false, &rc), ev);
         add_reader(*buf(R.keyB, g, false, &rc), ev);
+        if (R.keyC2 >= 0) add_reader(*buf(R.keyC2, g, false, &rc), ev);
         stats.tasks[g]++;
         stats.flops[g] += R.r.work;
     }
@@ -1009,6 +1017,12 @@ int Runtime::run_impl(const xk_call_t &call, bool wait) {
     }
     for (size_t g = 0; g < batch_.size(); ++g)
         if ((rc = flush_batch((int)g))) return rc;
+    if (call.routine == XK_ROUTINE_SYNC) {
+        // xk_sync: everything issued has completed (the API synchronised first), so tiles the
+        // planner dropped -- e.g. a call's shadow copies of C -- can go back to the pool
+        release_invalid();
+        return XK_OK;
+    }
     if (call.routine <= XK_ROUTINE_DTRSM && call.sync) {
         // the planner already passed its full sync point and invalidated the operands
         if ((rc = sync_all())) return rc;

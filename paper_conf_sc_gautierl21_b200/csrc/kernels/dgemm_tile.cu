@@ -228,9 +228,11 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
     cp_wait<0>();
 
     // epilogue: D = alpha*acc + beta*C (C not read when beta == 0)
-    const double alpha = t.alpha, beta = t.beta;
+    const double alpha = t.alpha, beta = t.beta, beta2 = t.beta2;
     double *C = t.C;
     const int64_t ldc = t.ldc;
+    const double *C2 = t.C2;
+    const int64_t ldc2 = t.ldc2;
 #pragma unroll
     for (int i = 0; i < MF; ++i) {
         const int64_t r = m0 + wm + i * 8 + fr;
@@ -245,6 +247,7 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
                 double *p = C + r + c * ldc;
                 double v = alpha * acc[i][j][h];
                 if (beta != 0.0) v = fma(beta, *p, v);
+                if (beta2 != 0.0) v = fma(beta2, C2[r + c * ldc2], v);
                 *p = v;
             }
         }
@@ -356,6 +359,9 @@ cudaError_t launch_dgemm_batch(bool ta, bool tb, TileBatch &b, cudaStream_t st) 
             u.alpha = t.alpha;
             u.beta = t.beta;
             u.tri = t.tri;
+            u.C2 = t.C2;
+            u.ldc2 = t.ldc2;
+            u.beta2 = t.beta2;
         }
         if (ok) return launch_dgemm_tma(ta, tb, tb_, st);
     }
@@ -384,7 +390,7 @@ cudaError_t launch_dgemm_tile(bool ta, bool tb, int64_t M, int64_t N, int64_t K,
     if (alpha == 0.0 || K <= 0) return launch_scale_tile(M, N, beta, C, ldc, st);
     TileBatch b;
     b.n = 1;
-    b.t[0] = TileTask{A, B, C, lda, ldb, ldc, M, N, K, alpha, beta, 0};
+    b.t[0] = TileTask{A, B, C, lda, ldb, ldc, M, N, K, alpha, beta, 0, nullptr, 0, 0.0};
     return launch_dgemm_batch(ta, tb, b, st);
 }
 

@@ -217,9 +217,11 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
     }
 
     // epilogue: D = alpha*acc + beta*C (C not read when beta == 0)
-    const double alpha = t.alpha, beta = t.beta;
+    const double alpha = t.alpha, beta = t.beta, beta2 = t.beta2;
     double *C = t.C;
     const int64_t ldc = t.ldc;
+    const double *C2 = t.C2;
+    const int64_t ldc2 = t.ldc2;
 #pragma unroll
     for (int i = 0; i < MF; ++i) {
         const int64_t r = m0 + wm + i * 8 + fr;
@@ -234,6 +236,7 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
                 double *p = C + r + c * ldc;
                 double v = alpha * acc[i][j][h];
                 if (beta != 0.0) v = fma(beta, *p, v);
+                if (beta2 != 0.0) v = fma(beta2, C2[r + c * ldc2], v);
                 *p = v;
             }
         }

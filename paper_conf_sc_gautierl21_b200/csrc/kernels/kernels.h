@@ -15,6 +15,9 @@ struct TileTask {
     int64_t M, N, K;
     double alpha, beta;
     int tri;  // 0 full tile; 1 / 2: write only the lower / upper triangle (SYRK diagonal tiles)
+    const double *C2 = nullptr;  // deferred beta: D += beta2 * C2 (beta2 == 0: C2 not read)
+    int64_t ldc2 = 0;
+    double beta2 = 0.0;
 };
 
 // A batch of independent tile tasks launched as one grid (grouped GEMM); passed by value
@@ -33,6 +36,9 @@ struct TmaTask {
     int64_t ldc, M, N, K;
     double alpha, beta;
     int tri;
+    const double *C2;
+    int64_t ldc2;
+    double beta2;
 };
 constexpr int kMaxTmaBatch = 16;
 struct TmaBatch {

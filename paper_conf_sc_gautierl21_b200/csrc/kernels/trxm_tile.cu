@@ -233,9 +233,9 @@ cudaError_t gemm_all(const TriOp &o, const Tiles &X, const Tiles &Y, const doubl
     tb.n = X.n;
     for (int q = 0; q < X.n; ++q) {
         if (o.left)
-            tb.t[q] = TileTask{P, X.B[q], Y.B[q], lda, X.ldb[q], Y.ldb[q], ny, X.other[q], nk, a, b, 0};
+            tb.t[q] = TileTask{P, X.B[q], Y.B[q], lda, X.ldb[q], Y.ldb[q], ny, X.other[q], nk, a, b, 0, nullptr, 0, 0.0};
         else
-            tb.t[q] = TileTask{X.B[q], P, Y.B[q], X.ldb[q], lda, Y.ldb[q], X.other[q], ny, nk, a, b, 0};
+            tb.t[q] = TileTask{X.B[q], P, Y.B[q], X.ldb[q], lda, Y.ldb[q], X.other[q], ny, nk, a, b, 0, nullptr, 0, 0.0};
     }
     return o.left ? launch_dgemm_batch(t, false, tb, st) : launch_dgemm_batch(false, t, tb, st);
 }

@@ -51,7 +51,7 @@ int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t
                                 std::string &err) {
     for (size_t i = 0; i < mats_.size(); ++i) {
         Matrix &M = mats_[i];
-        if (M.ld < 0) continue;  // forgotten
+        if (M.ld < 0 || M.shadow) continue;  // forgotten / per-call shadow
         if (M.base == base && M.ld == ld) {
             // tile extents must agree with the cached grid (step 9)
             int64_t T = flags_.T;
@@ -89,7 +89,7 @@ int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t
     uint64_t lo = base, hi = base + (uint64_t)((cols - 1) * ld + rows) * 8;
     for (size_t i = 0; i < mats_.size(); ++i) {
         Matrix &M = mats_[i];
-        if (M.ld < 0) continue;
+        if (M.ld < 0 || M.shadow) continue;
         uint64_t mlo = M.base, mhi = M.base + (uint64_t)((M.cols - 1) * M.ld + M.rows) * 8;
         if (lo < mhi && mlo < hi) {
             bool clean = true;
@@ -420,6 +420,8 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
         R.op = t.op;
         R.keyA = t.keyA;
         R.keyB = t.keyB;
+        R.keyC2 = t.keyC2;
+        R.beta2 = t.beta2;
         R.ta = t.ta;
         R.tb = t.tb;
         R.side = t.side;
@@ -472,6 +474,18 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
     }
     const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
     const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
+    // beta deferral (reading Q12''): when a C tile's input is valid on the host and its chain
+    // has >= 2 tasks, the first task does not read C (beta = 0) and the last one adds
+    // beta * C_input from a per-call shadow copy of the tile -- C crosses PCIe at the end of
+    // its chain, when the link is idle, instead of together with the first A/B tiles.  Tiles
+    // already valid on some GPU (data-on-device) are read in place as before
+    int ms = -1;
+    if (!scale_only && c.beta != 0.0 && tkn >= 2) {
+        Matrix S = mats_[mc];
+        S.shadow = true;
+        mats_.push_back(S);
+        ms = (int)mats_.size() - 1;
+    }
     Versions V;
     V.e = &entries_;
     std::vector<Task> tasks;
@@ -497,6 +511,11 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                 tasks.push_back(t);
                 continue;
             }
+            const Entry &ec = entries_[keyC];
+            bool defer = ms >= 0 && ec.host.present && ec.host.ver == ec.ver;
+            for (const NodeCopy &g : ec.gpu)  // already resident on a GPU: nothing to defer
+                if (g.present && g.ver == ec.ver) defer = false;
+            const int keyS = defer ? key_of(ms, i, j) : -1;
             for (int64_t kk = 0; kk < tkn; ++kk) {
                 int64_t kt = std::min(T, k - kk * T);
                 int keyA = ta ? key_of(ma, kk, i) : key_of(ma, i, kk);
@@ -507,29 +526,46 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                 t.out_key = keyC;
                 t.in.push_back({keyA, V.get(keyA), 0});
                 t.in.push_back({keyB, V.get(keyB), 1});
-                if (kk > 0 || c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                if (kk > 0 || (c.beta != 0.0 && !defer)) t.in.push_back({keyC, V.get(keyC), 2});
+                if (defer && kk == tkn - 1) {
+                    t.in.push_back({keyS, V.get(keyS), 2});
+                    t.keyC2 = keyS;
+                    t.beta2 = c.beta;
+                }
                 t.out_ver = V.bump(keyC);
                 t.keyA = keyA;
                 t.keyB = keyB;
                 t.ta = ta ? 'T' : 'N';
                 t.tb = tb ? 'T' : 'N';
                 t.alpha = c.alpha;
-                t.beta = (kk == 0) ? c.beta : 1.0;
+                t.beta = (kk == 0) ? (defer ? 0.0 : c.beta) : 1.0;
                 t.tk = kk;
                 t.i = i; t.j = j;
                 t.m = mt; t.n = nt; t.k = kt;
                 t.flops = 2 * mt * nt * kt;
                 // staggered k-chains (reading Q12'): tile (i,j) starts its chain at slot
-                // (i+j) mod tk, so chains begin and end at different times -- C's H2D spreads
-                // over the first tk slots and its D2H over the last ones instead of piling up
-                // at k = 0 and at the end
+                // (i+j) mod tk, so chains begin and end at different times and C's D2H
+                // spreads over the last tk slots instead of piling up at the end
                 int64_t sk[5] = {kk + (i + j) % tkn, (i + j + kk) % tmod, i, j, 0};
                 std::copy(sk, sk + 5, t.skey);
                 tasks.push_back(t);
             }
         }
     }
-    return run_tasks(tasks, c.sync != 0, out, err);
+    int rc = run_tasks(tasks, c.sync != 0, out, err);
+    if (ms >= 0) {
+        // the shadow tiles were only this call's inputs: drop their GPU copies and forget them
+        for (auto it = keymap_.begin(); it != keymap_.end();) {
+            if (entries_[it->second].mat == ms) {
+                for (auto &gc : entries_[it->second].gpu) gc.present = false;
+                it = keymap_.erase(it);
+            } else {
+                ++it;
+            }
+        }
+        mats_[ms].ld = -1;
+    }
+    return rc;
 }
 
 // DSYRK / DSYR2K (PLASMA pdsyrk / pdsyr2k): tiles of the uplo triangle of C; off-diagonal
@@ -870,7 +906,7 @@ bool Planner::view_tiles(uint64_t base, int64_t m, int64_t n, int64_t ld, int *m
                          int64_t *c0) const {
     for (size_t i = 0; i < mats_.size(); ++i) {
         const Matrix &M = mats_[i];
-        if (M.ld != ld || M.ld < 0) continue;
+        if (M.ld != ld || M.ld < 0 || M.shadow) continue;
         if (base < M.base) continue;
         uint64_t off = (base - M.base) / 8;
         int64_t rr = (int64_t)(off % (uint64_t)ld), cc = (int64_t)(off / (uint64_t)ld);

@@ -39,6 +39,7 @@ struct Matrix {
     uint64_t base = 0;
     int64_t ld = 0;
     int64_t rows = 0, cols = 0;  // stored extent covered by the tiles known so far
+    bool shadow = false;         // per-call read-only view of C's input values (beta deferral)
 };
 
 struct NodeCopy {
@@ -70,6 +71,8 @@ struct Rec {
     int tri = 0;                  // GEMM_TRI / SCALE on a diagonal tile: 1 lower, 2 upper
     double alpha = 1.0, beta = 0.0;
     int keyA = -1, keyB = -1;     // tiles in the kernel's A and B roles on dst (-1: none)
+    int keyC2 = -1;               // deferred-beta input tile: D += beta2 * C2 (-1: none)
+    double beta2 = 0.0;
     int64_t m = 0, n = 0, k = 0;  // task shape (output rows, cols, inner / triangle order)
 };
 
@@ -120,6 +123,8 @@ private:
         Inputs in;                  // inputs in position order (deps follow this order)
         int war = -1;               // readers slot of (out_key, out_ver - 1)
         int keyA = -1, keyB = -1;   // kernel roles
+        int keyC2 = -1;             // deferred beta: D += beta2 * (C's input tile)
+        double beta2 = 0.0;
         char ta = 'N', tb = 'N', side = 'L', uplo = 'L', diag = 'N';
         int tri = 0;
         double alpha = 1.0, beta = 0.0;

@@ -78,6 +78,7 @@ class Model:
         self.gfree = [0] * self.G
         self.hist = [[] for _ in range(self.G)]
         self.seq = 0
+        self.calls = 0
 
     # ------------------------------------------------------------------ helpers
     def owner(self, i, j):
@@ -176,6 +177,8 @@ class Model:
                 tasks = self.gen_trxm(routine == DTRSM, left, lower, ta, diag.upper(), m, n, alpha, A, lda, C, ldc)
             if tasks:
                 self.run(tasks, sync, out)
+            if routine == DGEMM:
+                self.drop_shadow(ldc)
             if sync and tasks is not None:
                 self.full_sync()
                 if routine == DGEMM:
@@ -231,6 +234,13 @@ class Model:
         tm, tn = ceil_div(m, T), ceil_div(n, T)
         tk = 0 if scale else ceil_div(k, T)
         tmod = max(1, tm, tn)
+        # beta deferral (Q12''): a per-call shadow of C's input tiles feeds the last
+        # task of each chain whose C input is valid on the host
+        shadow = None
+        if not scale and beta != 0 and tk >= 2:
+            self.calls += 1
+            shadow = ("shadow", self.calls, C)
+            self.extent[(shadow, ldc)] = list(self.extent[(C, ldc)])
         vers, tasks = {}, []
         for j in range(tn):
             for i in range(tm):
@@ -240,14 +250,29 @@ class Model:
                     ins = [(ct, 2)] if beta != 0 else []
                     tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
                     continue
+                defer = (shadow is not None and ct.host is not None and ct.host.ver == ct.ver
+                         and not any(g.ver == ct.ver for g in ct.gpus.values()))
+                st = self.tile(shadow, ldc, i, j) if defer else None
                 for kk in range(tk):
                     kt = min(T, k - kk * T)
                     at = self.tile(A, lda, kk, i) if ta else self.tile(A, lda, i, kk)
                     bt = self.tile(B, ldb, j, kk) if tb else self.tile(B, ldb, kk, j)
-                    ins = [(at, 0), (bt, 1)] + ([(ct, 2)] if (kk > 0 or beta != 0) else [])
+                    ins = [(at, 0), (bt, 1)] + ([(ct, 2)] if (kk > 0 or (beta != 0 and not defer)) else [])
+                    if defer and kk == tk - 1:
+                        ins.append((st, 2))
                     tasks.append(self._task(vers, OP_GEMM, i, j, ct, ins, (kk + (i + j) % tk, (i + j + kk) % tmod, i, j, 0),
                                             2 * mt * nt * kt, kk))
+        self._shadow = shadow
         return tasks
+
+    def drop_shadow(self, ldc):
+        sh = getattr(self, "_shadow", None)
+        if sh is None:
+            return
+        for key in [key for key in self.tiles if key[0] == sh]:
+            del self.tiles[key]
+        del self.extent[(sh, ldc)]
+        self._shadow = None
 
     def gen_syrk(self, two, lower, tr, n, k, alpha, beta, A, lda, B, ldb, C, ldc):
         if n == 0 or ((alpha == 0 or k == 0) and beta == 1):

@@ -354,3 +354,45 @@ def test_triangular_task_structure():
     # L tiles read: only the lower triangle of A is ever copied
     a_tiles = {(r[3], r[4]) for r in trsm if r[1] in (pm.H2D, pm.P2P) and r[2] == 0}
     assert all(i >= j for (i, j) in a_tiles) and len(a_tiles) == t * (t + 1) // 2
+
+
+def test_beta_deferral_structure():
+    """Reading Q12'': a host-valid C tile with a chain of >= 2 tasks is not read by the first
+    task (beta = 0, no C dependency); the last task adds beta*C from a shadow copy of the
+    original tile (4th dependency, an H2D of operand C at version 0).  C still crosses PCIe
+    exactly once per tile; a device-resident C (prefetched) is read in place, no deferral."""
+    T = 4
+    for G in (1, 4):
+        for t in (1, 2, 5):
+            N = t * T
+            call = xk.make_call(m=N, n=N, k=N, alpha=1.5, beta=-0.75, A=A_ADDR, lda=N, B=B_ADDR, ldb=N,
+                                C=C_ADDR, ldc=N, sync=True)
+            recs = xk.plan_dump(call, uniform(G), topo="ranked", optimistic=True, tile=T)
+            by_seq = {r[0]: r for r in recs}
+            tasks = [r for r in recs if r[1] == pm.TASK]
+            c_h2d = [r for r in recs if r[1] == pm.H2D and r[2] == 2]
+            assert len(c_h2d) == t * t and all(r[6] == 0 for r in c_h2d)
+            for r in tasks:
+                first, last = r[5] == 0, r[5] == t - 1
+                if t == 1:
+                    assert r[14][2] >= 0 and r[14][3] == -1
+                    continue
+                assert (r[14][2] == -1) == first
+                assert (r[14][3] >= 0) == last
+                if last:
+                    src = by_seq[r[14][3]]
+                    assert src[1] == pm.H2D and src[2] == 2 and (src[3], src[4]) == (r[3], r[4])
+            # the first task of every chain starts before its C tile finished crossing PCIe
+            if t >= 2:
+                late = sum(1 for r in tasks if r[5] == 0 and r[11] < by_seq[next(
+                    x[0] for x in c_h2d if (x[3], x[4]) == (r[3], r[4]))][12])
+                assert late > 0
+    # data-on-device: prefetched C is read in place
+    N, t = 20, 5
+    s = xk.PlanSession(uniform(2), topo="ranked", optimistic=True, tile=T)
+    s.call(xk.make_call(routine=pm.PREFETCH, m=N, n=N, C=C_ADDR, ldc=N, sync=False))
+    recs = s.call(xk.make_call(m=N, n=N, k=N, alpha=1.5, beta=-0.75, A=A_ADDR, lda=N, B=B_ADDR, ldb=N,
+                               C=C_ADDR, ldc=N, sync=False))
+    assert not any(r[1] == pm.H2D and r[2] == 2 for r in recs)
+    assert all(r[14][3] == -1 for r in recs if r[1] == pm.TASK)
+    s.close()
