@@ -87,6 +87,9 @@ int Runtime::init(const xk_config_t &cfg) {
         XK_CK(cudaStreamCreateWithFlags(&d.d2h, cudaStreamNonBlocking));
         XK_CK(cudaStreamCreateWithFlags(&d.p2p, cudaStreamNonBlocking));
         for (int k = 0; k < nks_; ++k) XK_CK(cudaStreamCreateWithFlags(&d.ks[k], cudaStreamNonBlocking));
+        int lo = 0, hi = 0;
+        XK_CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        XK_CK(cudaStreamCreateWithPriority(&d.kdiag, cudaStreamNonBlocking, hi));
     }
     cur_dev_ = -1;
     ev_pool_.assign(G, {});
@@ -341,6 +344,20 @@ int Runtime::issue(const Rec &R) {
     const Matrix &M = planner_->matrix(e.mat);
     const int64_t T = flags_.T;
     int rc = XK_OK;
+    // a record that depends on a deferred write-back: launch that batch (which issues it)
+    for (int q = 0; q < 4 && !deferred_seq_.empty(); ++q) {
+        auto it = r.dep[q] >= 0 ? deferred_seq_.find(r.dep[q]) : deferred_seq_.end();
+        if (it != deferred_seq_.end() && (rc = flush_batch(it->second))) return rc;
+    }
+    // the D2H of a tile whose last writer is still in this GPU's pending batch waits for the
+    // batch instead of launching it early (a step's diagonal ops / GEMMs stay one launch)
+    if (r.kind == XK_REC_D2H && r.dep[0] >= 0 && batch_[r.src].contains_seq(r.dep[0])) {
+        PendingBatch &bt = batch_[r.src];
+        bt.deferred.push_back(R);
+        bt.in_ids.push_back((int64_t)R.key * XK_MAX_GPUS + r.src);
+        deferred_seq_[r.seq] = r.src;
+        return XK_OK;
+    }
     if (r.kind != XK_REC_TASK && (rc = flush_for(R))) return rc;
     switch (r.kind) {
     case XK_REC_H2D: {
@@ -550,8 +567,12 @@ int Runtime::flush_batch(int g) {
     const Device &d = devs_[g];
     // kernel timing serialises the grouped launches on one stream so that each launch's
     // event-timed duration is its own (no overlap with a concurrent launch)
-    cudaStream_t s = kernel_timing ? d.ks[0] : d.ks[batch_count_[g]++ % cfg_.kstreams];
-    if (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG) {
+    const bool diag = bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG;
+    // diagonal-tile ops go to the high-priority stream: with the planner's lookahead (R9) a
+    // TRSM step's solve overlaps the previous step's trailing updates instead of queueing
+    // behind them
+    cudaStream_t s = kernel_timing ? d.ks[0] : diag ? d.kdiag : d.ks[batch_count_[g]++ % cfg_.kstreams];
+    if (diag) {
         const Rec &R0 = bt.recs[0];
         Buffer *A = buf(R0.keyA, g, false, &rc);
         if (!A) return rc;
@@ -598,7 +619,7 @@ int Runtime::flush_batch(int g) {
         bt.recs.clear();
         bt.out_ids.clear();
         bt.in_ids.clear();
-        return XK_OK;
+        return issue_deferred(g);
     }
     TileBatch tb;
     tb.n = (int)bt.recs.size();
@@ -655,6 +676,20 @@ int Runtime::flush_batch(int g) {
     bt.recs.clear();
     bt.out_ids.clear();
     bt.in_ids.clear();
+    return issue_deferred(g);
+}
+
+// Issue the write-backs that waited for GPU g's batch (now launched, so their last writer
+// has an event).
+int Runtime::issue_deferred(int g) {
+    if (batch_[g].deferred.empty()) return XK_OK;
+    std::vector<Rec> d;
+    d.swap(batch_[g].deferred);
+    for (const Rec &R : d) deferred_seq_.erase(R.r.seq);
+    for (const Rec &R : d) {
+        int rc = issue(R);
+        if (rc) return rc;
+    }
     return XK_OK;
 }
 
@@ -915,6 +950,7 @@ int Runtime::sync_all() {
         XK_CK(cudaStreamSynchronize(d.h2d));
         XK_CK(cudaStreamSynchronize(d.p2p));
         for (int k = 0; k < nks_; ++k) XK_CK(cudaStreamSynchronize(d.ks[k]));
+        XK_CK(cudaStreamSynchronize(d.kdiag));
         XK_CK(cudaStreamSynchronize(d.d2h));
     }
     cur_dev_ = -1;
@@ -1063,6 +1099,7 @@ int Runtime::finalize() {
         cudaStreamDestroy(d.d2h);
         cudaStreamDestroy(d.p2p);
         for (int k = 0; k < nks_; ++k) cudaStreamDestroy(d.ks[k]);
+        if (d.kdiag) cudaStreamDestroy(d.kdiag);
         for (cudaEvent_t e : ev_pool_[g]) cudaEventDestroy(e);
     }
     bufs_.clear();

@@ -40,6 +40,9 @@ struct Buffer {
 struct PendingBatch {
     std::vector<Rec> recs;  // copies (records are issued while they are planned)
     std::vector<int64_t> out_ids, in_ids;  // buffer ids written / read
+    // D2H write-backs of tiles this batch produces: issued right after the batch launches,
+    // so a write-back does not cut the batch short (their source ids are in in_ids)
+    std::vector<Rec> deferred;
     char ta = 'N', tb = 'N';
     int op = XK_OP_GEMM;  // GEMM / GEMM_TRI grouped launch, or TRSM_DIAG / TRMM_DIAG sharing keyA
     bool contains_seq(int64_t seq) const {
@@ -61,6 +64,7 @@ struct Device {
     int phys = 0;
     cudaStream_t h2d = nullptr, d2h = nullptr, p2p = nullptr;
     cudaStream_t ks[kMaxKStreams] = {};
+    cudaStream_t kdiag = nullptr;  // highest priority: diagonal-tile ops (critical path of TRSM)
     std::map<size_t, std::vector<double *>> free_bufs;  // caching allocator
     std::vector<std::pair<double *, size_t>> all_bufs;
     size_t bytes_in_use = 0;
@@ -98,6 +102,7 @@ private:
     int failed_ = 0;  // sticky runtime failure (XK_ERR_*), cleared by re-initialisation
     int issue(const Rec &r);
     int flush_batch(int g);
+    int issue_deferred(int g);
     int flush_for(const Rec &r);
     Buffer *buf(int key, int g, bool create, int *rc);
     void release_invalid();
@@ -144,6 +149,7 @@ private:
     std::map<uintptr_t, size_t> internal_reg_;  // registered by the library on first use
     int cur_dev_ = -1;
     std::vector<PendingBatch> batch_;
+    std::unordered_map<int64_t, int> deferred_seq_;  // seq of a deferred copy -> GPU of its batch
     std::vector<int64_t> batch_count_;
     std::vector<int64_t> batches_in_call_;  // grouped launches issued in the current call, per GPU
     int max_batch_ = kMaxBatch;

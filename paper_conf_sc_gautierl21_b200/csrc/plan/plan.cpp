@@ -893,7 +893,10 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
                 g.i = bi; g.j = bj;
                 g.m = mt; g.n = nt; g.k = kt;
                 g.flops = 2 * mt * nt * kt;
-                int64_t sk[5] = {s, 1, (bi + bj + s) % tmod, bi, bj};
+                // lookahead (reading R9): the row (col) the next step solves is updated first,
+                // so its diagonal solve can run while the other updates of this step proceed
+                const int64_t ph = (r == (fwd ? kx + 1 : kx - 1)) ? 1 : 2;
+                int64_t sk[5] = {s, ph, (bi + bj + s) % tmod, bi, bj};
                 std::copy(sk, sk + 5, g.skey);
                 tasks.push_back(g);
             }

@@ -413,7 +413,9 @@ class Model:
                         ins = [(opA(r, kx), 0), (self.tile(C, ldc, kx, bj), 2), (ot, 2)]
                     else:
                         ins = [(self.tile(C, ldc, bi, kx), 2), (opA(kx, r), 0), (ot, 2)]
-                    tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins, (s, 1, (bi + bj + s) % tmod, bi, bj),
+                    # lookahead (R9): the next step's row (column) is updated first
+                    ph = 1 if r == (kx + 1 if fwd else kx - 1) else 2
+                    tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins, (s, ph, (bi + bj + s) % tmod, bi, bj),
                                             2 * mt * nt * kt, s))
         return tasks
 

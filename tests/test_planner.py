@@ -396,3 +396,29 @@ def test_beta_deferral_structure():
     assert not any(r[1] == pm.H2D and r[2] == 2 for r in recs)
     assert all(r[14][3] == -1 for r in recs if r[1] == pm.TASK)
     s.close()
+
+
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_trsm_lookahead_order(uplo):
+    """Reading R9 (lookahead): in each step of the tiled TRSM the updates of the row the next
+    step solves come first, right after the step's diagonal solves, so the next diagonal
+    solve depends only on the first updates of the step."""
+    T, t = 4, 5
+    N = T * t
+    recs = xk.plan_dump(xk.make_call(routine=pm.DTRSM, side="L", uplo=uplo, transA="N", diag="N", m=N, n=N,
+                                     alpha=1.0, A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True), uniform(1), tile=T)
+    tasks = [r for r in recs if r[1] == pm.TASK]
+    order = list(range(t)) if uplo == "L" else list(range(t - 1, -1, -1))
+    pos = 0
+    for s, kx in enumerate(order):
+        diag = tasks[pos:pos + t]
+        assert all(r[15] == pm.OP_TRSM_DIAG and r[3] == kx for r in diag)
+        pos += t
+        nupd = t * (t - 1 - s)
+        upd = tasks[pos:pos + nupd]
+        assert all(r[15] == pm.OP_GEMM for r in upd)
+        if s + 1 < t:
+            assert all(r[3] == order[s + 1] for r in upd[:t])
+            assert all(r[3] != order[s + 1] for r in upd[t:])
+        pos += nupd
+    assert pos == len(tasks)
