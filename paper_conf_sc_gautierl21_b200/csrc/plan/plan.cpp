@@ -457,6 +457,40 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
 static bool is_t(char c) { return c == 'T' || c == 't' || c == 'C' || c == 'c'; }
 static char up(char c) { return (c >= 'a' && c <= 'z') ? (char)(c - 32) : c; }
 
+// beta deferral (reading Q12''): when a C tile's input is valid on the host only and its
+// chain has >= 2 tasks, the first task does not read C (beta = 0) and the last one adds
+// beta * C_input from a per-call shadow copy of the tile -- C crosses PCIe at the end of its
+// chain, when the link is idle, instead of together with the first A/B tiles.  Tiles
+// already valid on some GPU (data-on-device) are read in place as before.
+int Planner::add_shadow(int mc) {
+    Matrix S = mats_[mc];
+    S.shadow = true;
+    mats_.push_back(S);
+    return (int)mats_.size() - 1;
+}
+
+bool Planner::defer_beta(int keyC) const {
+    const Entry &ec = entries_[keyC];
+    if (!(ec.host.present && ec.host.ver == ec.ver)) return false;
+    for (const NodeCopy &g : ec.gpu)  // already resident on a GPU: nothing to defer
+        if (g.present && g.ver == ec.ver) return false;
+    return true;
+}
+
+// the shadow tiles were only this call's inputs: drop their GPU copies and forget them
+void Planner::drop_shadow(int ms) {
+    if (ms < 0) return;
+    for (auto it = keymap_.begin(); it != keymap_.end();) {
+        if (entries_[it->second].mat == ms) {
+            for (auto &gc : entries_[it->second].gpu) gc.present = false;
+            it = keymap_.erase(it);
+        } else {
+            ++it;
+        }
+    }
+    mats_[ms].ld = -1;
+}
+
 // DGEMM (PLASMA pdgemm structure): C(i,j) k-chains, beta on the first task.
 int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
     const int64_t m = c.m, n = c.n, k = c.k, T = flags_.T;
@@ -474,18 +508,7 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
     }
     const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
     const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
-    // beta deferral (reading Q12''): when a C tile's input is valid on the host and its chain
-    // has >= 2 tasks, the first task does not read C (beta = 0) and the last one adds
-    // beta * C_input from a per-call shadow copy of the tile -- C crosses PCIe at the end of
-    // its chain, when the link is idle, instead of together with the first A/B tiles.  Tiles
-    // already valid on some GPU (data-on-device) are read in place as before
-    int ms = -1;
-    if (!scale_only && c.beta != 0.0 && tkn >= 2) {
-        Matrix S = mats_[mc];
-        S.shadow = true;
-        mats_.push_back(S);
-        ms = (int)mats_.size() - 1;
-    }
+    const int ms = (!scale_only && c.beta != 0.0 && tkn >= 2) ? add_shadow(mc) : -1;
     Versions V;
     V.e = &entries_;
     std::vector<Task> tasks;
@@ -511,10 +534,7 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                 tasks.push_back(t);
                 continue;
             }
-            const Entry &ec = entries_[keyC];
-            bool defer = ms >= 0 && ec.host.present && ec.host.ver == ec.ver;
-            for (const NodeCopy &g : ec.gpu)  // already resident on a GPU: nothing to defer
-                if (g.present && g.ver == ec.ver) defer = false;
+            const bool defer = ms >= 0 && defer_beta(keyC);
             const int keyS = defer ? key_of(ms, i, j) : -1;
             for (int64_t kk = 0; kk < tkn; ++kk) {
                 int64_t kt = std::min(T, k - kk * T);
@@ -553,18 +573,7 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
         }
     }
     int rc = run_tasks(tasks, c.sync != 0, out, err);
-    if (ms >= 0) {
-        // the shadow tiles were only this call's inputs: drop their GPU copies and forget them
-        for (auto it = keymap_.begin(); it != keymap_.end();) {
-            if (entries_[it->second].mat == ms) {
-                for (auto &gc : entries_[it->second].gpu) gc.present = false;
-                it = keymap_.erase(it);
-            } else {
-                ++it;
-            }
-        }
-        mats_[ms].ld = -1;
-    }
+    drop_shadow(ms);
     return rc;
 }
 
@@ -591,6 +600,8 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
     const int64_t tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
     const int64_t tmod = std::max<int64_t>(1, tn);
     const int tri = lower ? 1 : 2;
+    const int64_t nchain = tkn * (two ? 2 : 1);  // tasks per C tile
+    const int ms = (!scale_only && c.beta != 0.0 && nchain >= 2) ? add_shadow(mc) : -1;
     Versions V;
     V.e = &entries_;
     std::vector<Task> tasks;
@@ -622,9 +633,13 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
                 continue;
             }
             bool first = true;
+            // diagonal tiles are always read in place (reading R5), off-diagonal ones defer beta
+            const bool defer = ms >= 0 && !dg && defer_beta(keyC);
+            const int keyS = defer ? key_of(ms, i, j) : -1;
+            int64_t pos = 0;
             for (int64_t l = 0; l < tkn; ++l) {
                 int64_t kt = std::min(T, k - l * T);
-                for (int s = 0; s < (two ? 2 : 1); ++s) {
+                for (int s = 0; s < (two ? 2 : 1); ++s, ++pos) {
                     // SYRK: op(A)_i op(A)_j^T.  SYR2K: s=0 op(A)_i op(B)_j^T, s=1 op(B)_i op(A)_j^T
                     int xa = (two && s == 1) ? mb : ma, xb = (two && s == 0) ? mb : ma;
                     int keyA = opnd(xa, i, l), keyB = opnd(xb, j, l);
@@ -635,19 +650,25 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
                     t.out_key = keyC;
                     t.in.push_back({keyA, V.get(keyA), xa == ma ? 0 : 1});
                     t.in.push_back({keyB, V.get(keyB), xb == ma ? 0 : 1});
-                    if (!first || c.beta != 0.0 || dg) t.in.push_back({keyC, V.get(keyC), 2});
+                    if (!first || (c.beta != 0.0 && !defer) || dg) t.in.push_back({keyC, V.get(keyC), 2});
+                    if (defer && pos == nchain - 1) {
+                        t.in.push_back({keyS, V.get(keyS), 2});
+                        t.keyC2 = keyS;
+                        t.beta2 = c.beta;
+                    }
                     t.out_ver = V.bump(keyC);
                     t.keyA = keyA;
                     t.keyB = keyB;
                     t.ta = tr ? 'T' : 'N';  // op(A) tile = X(i,l) or X(l,i)^T
                     t.tb = tr ? 'N' : 'T';  // op(B) tile = X(j,l)^T or X(l,j)
                     t.alpha = c.alpha;
-                    t.beta = first ? c.beta : 1.0;
+                    t.beta = first ? (defer ? 0.0 : c.beta) : 1.0;
                     t.tk = l;
                     t.i = i; t.j = j;
                     t.m = mt; t.n = nt; t.k = kt;
                     t.flops = dg ? kt * nt * (nt + 1) : 2 * mt * nt * kt;
-                    int64_t sk[5] = {2 * l + s, (i + j + l) % tmod, i, j, 0};
+                    // staggered chains (reading Q12'), as for DGEMM
+                    int64_t sk[5] = {2 * (l + (i + j) % tkn) + s, (i + j + l) % tmod, i, j, 0};
                     std::copy(sk, sk + 5, t.skey);
                     tasks.push_back(t);
                     first = false;
@@ -655,7 +676,9 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
             }
         }
     }
-    return run_tasks(tasks, c.sync != 0, out, err);
+    int rc = run_tasks(tasks, c.sync != 0, out, err);
+    drop_shadow(ms);
+    return rc;
 }
 
 // DSYMM (PLASMA pdsymm): C(i,j) k-chains over sym(A); the diagonal tile of A is used
@@ -678,6 +701,7 @@ int Planner::plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
     }
     const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tl = cdiv(ka, T);
     const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
+    const int ms = (!scale_only && c.beta != 0.0 && tl >= 2) ? add_shadow(mc) : -1;
     Versions V;
     V.e = &entries_;
     std::vector<Task> tasks;
@@ -702,6 +726,10 @@ int Planner::plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                 tasks.push_back(t);
                 continue;
             }
+            // beta deferral when the chain's last task is a GEMM (SYMM_DIAG reads C in place)
+            const bool last_diag = left ? (i == tl - 1) : (j == tl - 1);
+            const bool defer = ms >= 0 && !last_diag && defer_beta(keyC);
+            const int keyS = defer ? key_of(ms, i, j) : -1;
             for (int64_t l = 0; l < tl; ++l) {
                 int64_t kt = std::min(T, ka - l * T);
                 // sym(A) tile (r, q): stored (r, q) if it lies in the uplo triangle, else (q, r)^T
@@ -737,21 +765,29 @@ int Planner::plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
                     t.in.push_back({keyBt, V.get(keyBt), 1});
                     t.in.push_back({keyAt, V.get(keyAt), 0});
                 }
-                if (l > 0 || c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                if (l > 0 || (c.beta != 0.0 && !defer)) t.in.push_back({keyC, V.get(keyC), 2});
+                if (defer && l == tl - 1) {
+                    t.in.push_back({keyS, V.get(keyS), 2});
+                    t.keyC2 = keyS;
+                    t.beta2 = c.beta;
+                }
                 t.out_ver = V.bump(keyC);
                 t.alpha = c.alpha;
-                t.beta = (l == 0) ? c.beta : 1.0;
+                t.beta = (l == 0) ? (defer ? 0.0 : c.beta) : 1.0;
                 t.tk = l;
                 t.i = i; t.j = j;
                 t.m = mt; t.n = nt; t.k = kt;
                 t.flops = 2 * mt * nt * kt;
-                int64_t sk[5] = {l, (i + j + l) % tmod, i, j, 0};
+                // staggered chains (reading Q12'), as for DGEMM
+                int64_t sk[5] = {l + (i + j) % tl, (i + j + l) % tmod, i, j, 0};
                 std::copy(sk, sk + 5, t.skey);
                 tasks.push_back(t);
             }
         }
     }
-    return run_tasks(tasks, c.sync != 0, out, err);
+    int rc = run_tasks(tasks, c.sync != 0, out, err);
+    drop_shadow(ms);
+    return rc;
 }
 
 // DTRMM / DTRSM (PLASMA pdtrmm / pdtrsm) on the output B (passed as C).  op(A) is
@@ -832,10 +868,14 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             tasks.push_back(t);
             // TRMM: this tile's remaining contributions (sources still unmodified)
             if (!solve) {
+                // contributions nearest the diagonal first (reading R9): the one that reads
+                // the tile the next step overwrites comes first, so that step's diagonal
+                // multiply does not wait for this step's whole chain (WAR)
                 int64_t ph = 1;
-                for (int64_t q = 0; q < tk; ++q) {
-                    const bool contributes = left ? (elow ? q < kx : q > kx) : (elow ? q > kx : q < kx);
-                    if (!contributes) continue;
+                for (int64_t dq = 1; dq < tk; ++dq) {
+                    const bool below = left ? elow : !elow;  // contributing q lie below kx
+                    const int64_t q = below ? kx - dq : kx + dq;
+                    if (q < 0 || q >= tk) break;
                     int keyA_ = left ? opA(kx, q) : key_of(mc, bi, q);
                     int keyB_ = left ? key_of(mc, q, bj) : opA(q, kx);
                     const int64_t kt = std::min(T, ka - q * T);

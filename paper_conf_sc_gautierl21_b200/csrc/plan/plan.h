@@ -157,6 +157,10 @@ private:
     bool emit_copy(int key, int64_t ver, int d, int64_t treq, int operand, std::vector<Rec> &out);
     void emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, int64_t cols,
                   int64_t ready, int64_t dep, int operand, std::vector<Rec> &out);
+    // beta deferral (reading Q12''): per-call shadow view of C, its use, and its removal
+    int add_shadow(int mc);
+    bool defer_beta(int keyC) const;
+    void drop_shadow(int ms);
     int plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
     int plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std::string &err);
     int plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);

@@ -177,7 +177,7 @@ class Model:
                 tasks = self.gen_trxm(routine == DTRSM, left, lower, ta, diag.upper(), m, n, alpha, A, lda, C, ldc)
             if tasks:
                 self.run(tasks, sync, out)
-            if routine == DGEMM:
+            if routine in (DGEMM, DSYRK, DSYR2K, DSYMM):
                 self.drop_shadow(ldc)
             if sync and tasks is not None:
                 self.full_sync()
@@ -236,11 +236,7 @@ class Model:
         tmod = max(1, tm, tn)
         # beta deferral (Q12''): a per-call shadow of C's input tiles feeds the last
         # task of each chain whose C input is valid on the host
-        shadow = None
-        if not scale and beta != 0 and tk >= 2:
-            self.calls += 1
-            shadow = ("shadow", self.calls, C)
-            self.extent[(shadow, ldc)] = list(self.extent[(C, ldc)])
+        shadow = self.new_shadow(C, ldc) if (not scale and beta != 0 and tk >= 2) else None
         vers, tasks = {}, []
         for j in range(tn):
             for i in range(tm):
@@ -250,8 +246,7 @@ class Model:
                     ins = [(ct, 2)] if beta != 0 else []
                     tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
                     continue
-                defer = (shadow is not None and ct.host is not None and ct.host.ver == ct.ver
-                         and not any(g.ver == ct.ver for g in ct.gpus.values()))
+                defer = shadow is not None and self.host_only(ct)
                 st = self.tile(shadow, ldc, i, j) if defer else None
                 for kk in range(tk):
                     kt = min(T, k - kk * T)
@@ -264,6 +259,18 @@ class Model:
                                             2 * mt * nt * kt, kk))
         self._shadow = shadow
         return tasks
+
+    def new_shadow(self, C, ldc):
+        self.calls += 1
+        shadow = ("shadow", self.calls, C)
+        self.extent[(shadow, ldc)] = list(self.extent[(C, ldc)])
+        self._shadow = shadow
+        return shadow
+
+    @staticmethod
+    def host_only(ct):
+        return (ct.host is not None and ct.host.ver == ct.ver
+                and not any(g.ver == ct.ver for g in ct.gpus.values()))
 
     def drop_shadow(self, ldc):
         sh = getattr(self, "_shadow", None)
@@ -287,6 +294,8 @@ class Model:
         tn = ceil_div(n, T)
         tk = 0 if scale else ceil_div(k, T)
         tmod = max(1, tn)
+        nchain = tk * (2 if two else 1)
+        shadow = self.new_shadow(C, ldc) if (not scale and beta != 0 and nchain >= 2) else None
         vers, tasks = {}, []
 
         def opnd(X, ld, r, l):
@@ -303,17 +312,23 @@ class Model:
                     tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
                     continue
                 first = True
+                defer = shadow is not None and not dg and self.host_only(ct)  # diagonal: R5
+                pos = 0
                 for l in range(tk):
                     kt = min(T, k - l * T)
                     for s in range(2 if two else 1):
                         xa = (B, ldb, 1) if (two and s == 1) else (A, lda, 0)
                         xb = (B, ldb, 1) if (two and s == 0) else (A, lda, 0)
                         at, bt = opnd(xa[0], xa[1], i, l), opnd(xb[0], xb[1], j, l)
-                        ins = [(at, xa[2]), (bt, xb[2])] + ([(ct, 2)] if (not first or beta != 0 or dg) else [])
+                        ins = [(at, xa[2]), (bt, xb[2])] + (
+                            [(ct, 2)] if (not first or (beta != 0 and not defer) or dg) else [])
+                        if defer and pos == nchain - 1:
+                            ins.append((self.tile(shadow, ldc, i, j), 2))
                         fl = kt * nt * (nt + 1) if dg else 2 * mt * nt * kt
                         tasks.append(self._task(vers, OP_GEMM_TRI if dg else OP_GEMM, i, j, ct, ins,
-                                                (2 * l + s, (i + j + l) % tmod, i, j, 0), fl, l))
+                                                (2 * (l + (i + j) % tk) + s, (i + j + l) % tmod, i, j, 0), fl, l))
                         first = False
+                        pos += 1
         return tasks
 
     def gen_symm(self, left, lower, m, n, alpha, beta, A, lda, B, ldb, C, ldc):
@@ -328,6 +343,7 @@ class Model:
             self.matrix(B, ldb, m, n)
         tm, tn, tl = ceil_div(m, T), ceil_div(n, T), ceil_div(ka, T)
         tmod = max(1, tm, tn)
+        shadow = self.new_shadow(C, ldc) if (not scale and beta != 0 and tl >= 2) else None
         vers, tasks = {}, []
         for j in range(tn):
             for i in range(tm):
@@ -337,6 +353,8 @@ class Model:
                     ins = [(ct, 2)] if beta != 0 else []
                     tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
                     continue
+                last_diag = (i == tl - 1) if left else (j == tl - 1)  # SYMM_DIAG reads C in place
+                defer = shadow is not None and not last_diag and self.host_only(ct)
                 for l in range(tl):
                     kt = min(T, ka - l * T)
                     r, q = (i, l) if left else (l, j)
@@ -347,10 +365,12 @@ class Model:
                         ins = [(at, 0), (bt, 1)]
                     else:
                         ins = [(bt, 1), (at, 0)]
-                    if l > 0 or beta != 0:
+                    if l > 0 or (beta != 0 and not defer):
                         ins.append((ct, 2))
+                    if defer and l == tl - 1:
+                        ins.append((self.tile(shadow, ldc, i, j), 2))
                     tasks.append(self._task(vers, OP_SYMM_DIAG if r == q else OP_GEMM, i, j, ct, ins,
-                                            (l, (i + j + l) % tmod, i, j, 0), 2 * mt * nt * kt, l))
+                                            (l + (i + j) % tl, (i + j + l) % tmod, i, j, 0), 2 * mt * nt * kt, l))
         return tasks
 
     def gen_trxm(self, solve, left, lower, tr, diag, m, n, alpha, A, lda, C, ldc):
@@ -387,10 +407,10 @@ class Model:
                                         [(opA(kx, kx), 0), (ot, 2)], (s, 0, (bi + bj + s) % tmod, bi, bj), fl, s))
                 if not solve:
                     ph = 1
-                    for q in range(tk):
-                        contrib = (q < kx if elow else q > kx) if left else (q > kx if elow else q < kx)
-                        if not contrib:
-                            continue
+                    # contributions nearest the diagonal first (R9)
+                    below = elow if left else not elow
+                    qs = range(kx - 1, -1, -1) if below else range(kx + 1, tk)
+                    for q in qs:
                         kt = min(T, ka - q * T)
                         if left:
                             ins = [(opA(kx, q), 0), (self.tile(C, ldc, q, bj), 2), (ot, 2)]

@@ -422,3 +422,53 @@ def test_trsm_lookahead_order(uplo):
             assert all(r[3] != order[s + 1] for r in upd[t:])
         pos += nupd
     assert pos == len(tasks)
+
+
+def test_trmm_contributions_nearest_first():
+    """Reading R9 for TRMM (in place, bottom-up for left/lower): the contributions to
+    B(kx, o) run nearest the diagonal first (q = kx-1, kx-2, ...), so the next step's
+    diagonal multiply on row kx-1 waits only for the first contribution of each chain
+    (the WAR on B(kx-1, o)), not for the whole step."""
+    T, t = 4, 5
+    N = T * t
+    recs = xk.plan_dump(xk.make_call(routine=pm.DTRMM, side="L", uplo="L", transA="N", diag="N", m=N, n=N,
+                                     alpha=1.0, A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True), uniform(1), tile=T)
+    by_seq = {r[0]: r for r in recs}
+    qs = {}
+    for r in recs:
+        if r[1] == pm.TASK and r[15] == pm.OP_GEMM:
+            a = by_seq[r[14][0]]  # producer of the A tile read: H2D of A(kx, q)
+            assert a[1] == pm.H2D and a[2] == 0 and a[3] == r[3]
+            qs.setdefault((r[3], r[4]), []).append(a[4])
+    assert len(qs) == t * (t - 1)
+    for (kx, o), q in qs.items():
+        assert q == list(range(kx - 1, -1, -1)), (kx, o, q)
+
+
+def test_beta_deferral_syrk_symm():
+    """Reading Q12'' extended to DSYRK/DSYR2K/DSYMM: off-diagonal SYRK tiles and SYMM tiles
+    whose chain ends in a GEMM defer beta to the last task (shadow H2D of C, operand 2,
+    version 0); SYRK diagonal tiles (reading R5) and SYMM chains ending in the symmetric
+    diagonal op read C in place.  C still crosses PCIe once per tile."""
+    T, t = 4, 3
+    N = T * t
+    for routine in (pm.DSYRK, pm.DSYR2K, pm.DSYMM):
+        call = xk.make_call(routine=routine, uplo="L", transA="N", side="L", m=N, n=N, k=N, alpha=1.5,
+                            beta=-0.75, A=A_ADDR, lda=N, B=B_ADDR, ldb=N, C=C_ADDR, ldc=N, sync=True)
+        recs = xk.plan_dump(call, uniform(2), tile=T)
+        by_seq = {r[0]: r for r in recs}
+        chains = {}
+        for r in recs:
+            if r[1] == pm.TASK:
+                chains.setdefault((r[3], r[4]), []).append(r)
+        c_h2d = [r for r in recs if r[1] == pm.H2D and r[2] == 2]
+        assert len(c_h2d) == len(chains)
+        for (i, j), ch in chains.items():
+            in_place = (i == j) if routine != pm.DSYMM else (i == t - 1)
+            first, last = ch[0], ch[-1]
+            if in_place:
+                assert all(d == -1 for d in last[14][3:]) and first[14][2] >= 0
+            else:
+                assert first[14][2] == -1
+                src = by_seq[last[14][3]]
+                assert src[1] == pm.H2D and src[2] == 2 and (src[3], src[4]) == (i, j)
