@@ -37,13 +37,20 @@ struct BaseBatch {
     int64_t ldb[kMaxBatch], nvec[kMaxBatch];
 };
 
+constexpr int LDM = NB + 2;  // triangle stride in shared memory (16-byte aligned rows)
+
 template <bool SOLVE, bool LOWER, bool LEFT>
 __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ BaseBatch bb, int n,
                                                        double alpha, const double *A, int64_t lda,
                                                        bool mtrans, bool unit) {
     extern __shared__ double sm[];
-    double(*Ms)[NB + 1] = reinterpret_cast<double(*)[NB + 1]>(sm);
-    double(*V)[NB + 1] = reinterpret_cast<double(*)[NB + 1]>(sm + NB * (NB + 1));  // V[element][vector]
+    // SOLVE: Ms[c * LDM + i] = M(i, c) (columns contiguous: column-oriented substitution);
+    // multiply: Ms[i * LDM + c] = M(i, c) (rows contiguous: row dot products).  Either way
+    // the inner loop reads two consecutive entries with one 16-byte shared load, and every
+    // thread of the warp reads the same address (broadcast).
+    double *Ms = sm;
+    double(*V)[NB + 1] = reinterpret_cast<double(*)[NB + 1]>(sm + NB * LDM);  // V[element][vector]
+    double *rd = sm + NB * LDM + NB * (NB + 1);                               // 1 / M(l, l)
     int q = 0;
 #pragma unroll 1
     while (q + 1 < bb.n && (int)blockIdx.x >= bb.cta_start[q + 1]) ++q;
@@ -52,42 +59,41 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ B
     const int64_t es = LEFT ? 1 : ldb, vs = LEFT ? ldb : 1;
     const int tid = threadIdx.x;
     const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * NB;
-    // triangle of M into shared memory (only the referenced part is read); the load loops
-    // are unrolled so many global loads are in flight per thread (the kernel is latency-bound)
-#pragma unroll 16
-    for (int r = tid; r < n * n; r += NB) {
-        int i = r % n, c = r / n;
-        bool in = LOWER ? (i > c) : (i < c);
-        double x = 0.0;
-        if (in) x = opa(A, lda, mtrans, i, c);
-        else if (i == c) x = unit ? 1.0 : opa(A, lda, mtrans, i, c);
-        Ms[i][c] = x;
-    }
-    // vectors of this CTA (coalesced along the contiguous direction)
+    // triangle of M into shared memory, padded to NB with the identity (only the referenced
+    // part of A is read).  The kernel is latency-bound, so every load of a phase is issued
+    // before the first shared store (fully unrolled, one element per thread per column:
+    // coalesced along the stored-contiguous direction of A for either transposition).
     const int nv = (int)((nvec - v0) < NB ? (nvec - v0) : NB);
-    if (LEFT) {
-#pragma unroll 16
-        for (int r = tid; r < n * nv; r += NB) {
-            int e = r % n, v = r / n;
-            V[e][v] = B[e + (v0 + v) * vs];
+    {
+        double t[NB];
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            const int i = mtrans ? k : tid, c = mtrans ? tid : k;  // M(i, c); A contiguous in tid
+            const bool in = LOWER ? (i > c) : (i < c);
+            double x = (i == c) ? 1.0 : 0.0;
+            if (i < n && c < n && (in || (i == c && !unit))) x = opa(A, lda, mtrans, i, c);
+            t[k] = x;
         }
-    } else {
-#pragma unroll 16
-        for (int r = tid; r < n * nv; r += NB) {
-            int v = r % nv, e = r / nv;
-            V[e][v] = B[(v0 + v) * vs + e * es];
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            const int i = mtrans ? k : tid, c = mtrans ? tid : k;
+            Ms[SOLVE ? c * LDM + i : i * LDM + c] = t[k];
+            if (SOLVE && i == c) rd[i] = 1.0 / t[k];
         }
-    }
-    // pad the triangle to NB with the identity and the vectors with zeros, so the fully
-    // unrolled register code below always works on NB x NB (padded rows stay zero and are
-    // never stored)
-    for (int r = tid; r < NB * NB; r += NB) {
-        int i = r % NB, c = r / NB;
-        if (i >= n || c >= n) Ms[i][c] = (i == c) ? 1.0 : 0.0;
-    }
-    for (int r = tid; r < NB * NB; r += NB) {
-        int e = r % NB, v = r / NB;
-        if (e >= n || v >= nv) V[e][v] = 0.0;
+        // vectors of this CTA (coalesced along the contiguous direction of B), zero-padded
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            if (LEFT) {  // element e = tid of vector k
+                t[k] = (tid < n && k < nv) ? B[tid + (v0 + k) * vs] : 0.0;
+            } else {     // vector tid, element k
+                t[k] = (k < n && tid < nv) ? B[(v0 + tid) * vs + k * es] : 0.0;
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            if (LEFT) V[tid][k] = t[k];
+            else V[k][tid] = t[k];
+        }
     }
     __syncthreads();
     {
@@ -103,33 +109,53 @@ __global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ B
             if (LOWER) {  // column-oriented forward substitution: x_i -= M_il x_l, l ascending
 #pragma unroll
                 for (int l = 0; l < NB; ++l) {
-                    if (!unit) x[l] = x[l] / Ms[l][l];
+                    if (!unit) x[l] *= rd[l];
+                    const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
 #pragma unroll
-                    for (int i = l + 1; i < NB; ++i) x[i] -= Ms[i][l] * x[l];
+                    for (int p = (l + 1) / 2; p < NB / 2; ++p) {
+                        const double2 m2 = col[p];
+                        if (2 * p > l) x[2 * p] -= m2.x * x[l];
+                        x[2 * p + 1] -= m2.y * x[l];
+                    }
                 }
             } else {      // back substitution, l descending
 #pragma unroll
                 for (int l = NB - 1; l >= 0; --l) {
-                    if (!unit) x[l] = x[l] / Ms[l][l];
+                    if (!unit) x[l] *= rd[l];
+                    const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
 #pragma unroll
-                    for (int i = 0; i < l; ++i) x[i] -= Ms[i][l] * x[l];
+                    for (int p = 0; 2 * p < l; ++p) {
+                        const double2 m2 = col[p];
+                        x[2 * p] -= m2.x * x[l];
+                        if (2 * p + 1 < l) x[2 * p + 1] -= m2.y * x[l];
+                    }
                 }
             }
         } else {
             if (LOWER) {  // bottom-up: row i only reads x_0..x_i, still unmodified
 #pragma unroll
                 for (int i = NB - 1; i >= 0; --i) {
+                    const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
                     double s = 0.0;
 #pragma unroll
-                    for (int l = 0; l <= i; ++l) s += Ms[i][l] * x[l];
+                    for (int p = 0; 2 * p <= i; ++p) {
+                        const double2 m2 = row[p];
+                        s += m2.x * x[2 * p];
+                        if (2 * p + 1 <= i) s += m2.y * x[2 * p + 1];
+                    }
                     x[i] = alpha * s;
                 }
-            } else {
+            } else {      // top-down: row i only reads x_i..x_NB-1, still unmodified
 #pragma unroll
                 for (int i = 0; i < NB; ++i) {
+                    const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
                     double s = 0.0;
 #pragma unroll
-                    for (int l = i; l < NB; ++l) s += Ms[i][l] * x[l];
+                    for (int p = i / 2; p < NB / 2; ++p) {
+                        const double2 m2 = row[p];
+                        if (2 * p >= i) s += m2.x * x[2 * p];
+                        s += m2.y * x[2 * p + 1];
+                    }
                     x[i] = alpha * s;
                 }
             }
@@ -175,7 +201,7 @@ inline const double *opa_block(const double *A, int64_t lda, bool trans, int64_t
 template <bool SOLVE, bool LOWER, bool LEFT>
 cudaError_t base_launch(const BaseBatch &bb, unsigned grid, int n, double alpha, const double *A,
                         int64_t lda, bool mtrans, bool unit, cudaStream_t st) {
-    constexpr size_t smem = 2 * NB * (NB + 1) * sizeof(double);
+    constexpr size_t smem = (NB * LDM + NB * (NB + 1) + NB) * sizeof(double);
     auto kern = trxm_base_kernel<SOLVE, LOWER, LEFT>;
     static unsigned attr_set = 0;  // per instantiation, one bit per device
     int dev = 0;
