@@ -61,9 +61,15 @@ def parse():
 
 
 # --------------------------------------------------------------------------- distributed
+_HOST_GROUP = None  # gloo group for barriers / timing reductions: host-side waits only
+
+
 def dist_setup(backend=None):
     """One process per GPU under torchrun (RANK/LOCAL_RANK/WORLD_SIZE/MASTER_* from the env).
-    backend: "nccl" on GPU boxes (default), "gloo" for the CPU tests of this path."""
+    backend: "nccl" on GPU boxes (default), "gloo" for the CPU tests of this path.
+    The barriers and the max-over-ranks reduction go through a gloo group: a rank waiting in
+    a barrier must not park an NCCL kernel on its GPU while rank 0's library computes on it."""
+    global _HOST_GROUP
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     if ws > 1:
@@ -75,15 +81,17 @@ def dist_setup(backend=None):
             lr = int(os.environ.get("LOCAL_RANK", rank))
             torch.cuda.set_device(lr)
             dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+            _HOST_GROUP = dist.new_group(backend="gloo")
         else:
             dist.init_process_group(backend)
+            _HOST_GROUP = dist.group.WORLD
     return rank, ws
 
 
 def barrier(ws):
     if ws > 1:
         import torch.distributed as dist
-        dist.barrier()
+        dist.barrier(group=_HOST_GROUP)
 
 
 def max_over_ranks(x, ws):
@@ -93,9 +101,8 @@ def max_over_ranks(x, ws):
         return x
     import torch
     import torch.distributed as dist
-    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
-    t = torch.tensor([x], dtype=torch.float64, device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    t = torch.tensor([x], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=_HOST_GROUP)
     return float(t.item())
 
 
@@ -387,7 +394,7 @@ def main():
         run_xk(args, rank, ws)
     if ws > 1:
         import torch.distributed as dist
-        dist.barrier()
+        barrier(ws)
         dist.destroy_process_group()
 
 
