@@ -66,6 +66,10 @@ int Runtime::init(const xk_config_t &cfg) {
     }
     int ks = cfg.kstreams > 0 ? std::min(cfg.kstreams, kMaxKStreams) : 2;
     cfg_.kstreams = ks;
+    {
+        const char *dv = getenv("XK_DEFER_D2H");
+        defer_d2h_ = !(dv && dv[0] == '0');
+    }
     nks_ = std::max(ks, 4);  // streams created: batches use the first ks, diagonal ops all
     // peer access between distinct physical devices (NVLink / NVSwitch)
     for (int a = 0; a < G; ++a)
@@ -350,8 +354,10 @@ int Runtime::issue(const Rec &R) {
         if (it != deferred_seq_.end() && (rc = flush_batch(it->second))) return rc;
     }
     // the D2H of a tile whose last writer is still in this GPU's pending batch waits for the
-    // batch instead of launching it early (a step's diagonal ops / GEMMs stay one launch)
-    if (r.kind == XK_REC_D2H && r.dep[0] >= 0 && batch_[r.src].contains_seq(r.dep[0])) {
+    // batch instead of launching it early (a step's diagonal ops / GEMMs stay one launch) --
+    // except in the GPU's last tasks of the call, where the write-back is the tail
+    if (defer_d2h_ && r.kind == XK_REC_D2H && r.dep[0] >= 0 && batch_[r.src].contains_seq(r.dep[0]) &&
+        batch_[r.src].recs.back().remaining >= max_batch_) {
         PendingBatch &bt = batch_[r.src];
         bt.deferred.push_back(R);
         bt.in_ids.push_back((int64_t)R.key * XK_MAX_GPUS + r.src);
@@ -509,7 +515,11 @@ int Runtime::issue(const Rec &R) {
         // batch size ramps 1, 2, 4, ... up to max_batch_ at the start of each call, so the
         // first kernels start as soon as their own inputs have landed instead of waiting
         // for a whole batch worth of tiles to cross PCIe
-        const int cap = (int)std::min<int64_t>(max_batch_, (int64_t)1 << std::min<int64_t>(batches_in_call_[g], 5));
+        // ... and ramps down (half of the GPU's remaining tasks) at the end, so the write-back
+        // of the last C tiles does not wait for one large final batch
+        const int64_t left0 = (bt.recs.empty() ? R.remaining : bt.recs[0].remaining) + 1;
+        const int cap = (int)std::min<int64_t>(std::min<int64_t>(max_batch_, std::max<int64_t>(1, (left0 + 1) / 2)),
+                                               (int64_t)1 << std::min<int64_t>(batches_in_call_[g], 5));
         bool conflict = (int)bt.recs.size() >= cap ||
                         (!bt.recs.empty() && (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG)) ||
                         (!bt.recs.empty() && (bt.ta != R.ta || bt.tb != R.tb)) ||

@@ -433,6 +433,7 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
         R.m = t.m;
         R.n = t.n;
         R.k = t.k;
+        R.remaining = (int64_t)(lists[d].size() - pos[d]) - 1;
         emit(R, out);
         if (sink_rc_) {
             err = "issue failed";

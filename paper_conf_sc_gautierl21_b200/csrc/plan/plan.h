@@ -74,6 +74,7 @@ struct Rec {
     int keyC2 = -1;               // deferred-beta input tile: D += beta2 * C2 (-1: none)
     double beta2 = 0.0;
     int64_t m = 0, n = 0, k = 0;  // task shape (output rows, cols, inner / triangle order)
+    int64_t remaining = 0;        // TASK: tasks after this one on its GPU in this call
 };
 
 class Planner {
