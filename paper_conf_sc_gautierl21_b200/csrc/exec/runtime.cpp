@@ -69,6 +69,8 @@ int Runtime::init(const xk_config_t &cfg) {
     {
         const char *dv = getenv("XK_DEFER_D2H");
         defer_d2h_ = !(dv && dv[0] == '0');
+        const char *rv = getenv("XK_RAMP");  // grouped launches per batch-size doubling
+        ramp_div_ = rv ? std::max(1, atoi(rv)) : ramp_div_;
     }
     nks_ = std::max(ks, 4);  // streams created: batches use the first ks, diagonal ops all
     // peer access between distinct physical devices (NVLink / NVSwitch)
@@ -512,14 +514,15 @@ int Runtime::issue(const Rec &R) {
         const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g, idB = (int64_t)R.keyB * XK_MAX_GPUS + g;
         const int64_t idC2 = R.keyC2 >= 0 ? (int64_t)R.keyC2 * XK_MAX_GPUS + g : -1;
         PendingBatch &bt = batch_[g];
-        // batch size ramps 1, 2, 4, ... up to max_batch_ at the start of each call, so the
+        // batch size ramps 1, 2, 4, ... (ramp_div_ launches per size, XK_RAMP) up to max_batch_
+        // at the start of each call, so the
         // first kernels start as soon as their own inputs have landed instead of waiting
         // for a whole batch worth of tiles to cross PCIe
         // ... and ramps down (half of the GPU's remaining tasks) at the end, so the write-back
         // of the last C tiles does not wait for one large final batch
         const int64_t left0 = (bt.recs.empty() ? R.remaining : bt.recs[0].remaining) + 1;
         const int cap = (int)std::min<int64_t>(std::min<int64_t>(max_batch_, std::max<int64_t>(1, (left0 + 1) / 2)),
-                                               (int64_t)1 << std::min<int64_t>(batches_in_call_[g], 5));
+                                               (int64_t)1 << std::min<int64_t>(batches_in_call_[g] / ramp_div_, 5));
         bool conflict = (int)bt.recs.size() >= cap ||
                         (!bt.recs.empty() && (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG)) ||
                         (!bt.recs.empty() && (bt.ta != R.ta || bt.tb != R.tb)) ||

@@ -149,8 +149,9 @@ private:
     std::map<uintptr_t, size_t> internal_reg_;  // registered by the library on first use
     int cur_dev_ = -1;
     std::vector<PendingBatch> batch_;
-    std::unordered_map<int64_t, int> deferred_seq_;
-    bool defer_d2h_ = true;  // XK_DEFER_D2H=0: a write-back launches its batch at once  // seq of a deferred copy -> GPU of its batch
+    std::unordered_map<int64_t, int> deferred_seq_;  // seq of a deferred copy -> GPU of its batch
+    bool defer_d2h_ = true;  // XK_DEFER_D2H=0: a write-back launches its batch at once
+    int ramp_div_ = 8;       // batch size doubles every ramp_div_ launches at a call's start (XK_RAMP)
     std::vector<int64_t> batch_count_;
     std::vector<int64_t> batches_in_call_;  // grouped launches issued in the current call, per GPU
     int max_batch_ = kMaxBatch;
