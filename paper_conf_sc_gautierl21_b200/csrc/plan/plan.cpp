@@ -992,6 +992,14 @@ int Planner::plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::strin
     if (!view_tiles(c.C, c.m, c.n, (int64_t)c.ldc, &mat, &r0, &c0)) return XK_OK;  // never cached
     const Matrix &M = mats_[mat];
     int64_t rend = std::min(M.rows, r0 + c.m), cend = std::min(M.cols, c0 + c.n);
+    // write-backs go out in the (virtual) completion order of their tiles, so the FIFO D2H
+    // stream is never held by a tile whose chain ends late (ties: column-major tile order)
+    struct WB {
+        int64_t t_done;
+        int key, src;
+        int64_t r0, c0, rows, cols;
+    };
+    std::vector<WB> wb;
     for (int64_t bj = c0 / T; bj * T < cend; ++bj) {
         for (int64_t bi = r0 / T; bi * T < rend; ++bi) {
             auto it = keymap_.find(tile_key(mat, bi, bj));
@@ -1012,9 +1020,13 @@ int Planner::plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::strin
             int64_t tr1 = std::min(rend, bi * T + e.rows) - bi * T;
             int64_t tc1 = std::min(cend, bj * T + e.cols) - bj * T;
             if (tr1 <= tr0 || tc1 <= tc0) continue;
-            emit_d2h(it->second, src, tr0, tc0, tr1 - tr0, tc1 - tc0, e.gpu[src].t_done,
-                     e.gpu[src].producer, 2, out);
+            wb.push_back({e.gpu[src].t_done, it->second, src, tr0, tc0, tr1 - tr0, tc1 - tc0});
         }
+    }
+    std::stable_sort(wb.begin(), wb.end(), [](const WB &a, const WB &b) { return a.t_done < b.t_done; });
+    for (const WB &w : wb) {
+        const Entry &e = entries_[w.key];
+        emit_d2h(w.key, w.src, w.r0, w.c0, w.rows, w.cols, w.t_done, e.gpu[w.src].producer, 2, out);
     }
     return XK_OK;
 }

@@ -526,6 +526,7 @@ class Model:
         b, r0, c0, rows, cols = loc
         T = self.T
         rend, cend = min(rows, r0 + m), min(cols, c0 + n)
+        wb = []
         for bj in range(c0 // T, ceil_div(cend, T)):
             for bi in range(r0 // T, ceil_div(rend, T)):
                 t = self.tiles.get((b, ld, bi, bj))
@@ -537,8 +538,11 @@ class Model:
                 tr1, tc1 = min(rend, bi * T + t.rows) - bi * T, min(cend, bj * T + t.cols) - bj * T
                 if tr1 <= tr0 or tc1 <= tc0:
                     continue
-                self.copy_out(t, src, (tr0, tc0, tr1 - tr0, tc1 - tc0), t.gpus[src].t_done,
-                              t.gpus[src].producer, out)
+                wb.append((t, src, (tr0, tc0, tr1 - tr0, tc1 - tc0)))
+        # write-backs in completion order of their tiles (stable: column-major ties)
+        wb.sort(key=lambda w: w[0].gpus[w[1]].t_done)
+        for t, src, sub in wb:
+            self.copy_out(t, src, sub, t.gpus[src].t_done, t.gpus[src].producer, out)
 
     def prefetch(self, base, m, n, ld, out):
         if m <= 0 or n <= 0:

@@ -472,3 +472,19 @@ def test_beta_deferral_syrk_symm():
                 assert first[14][2] == -1
                 src = by_seq[last[14][3]]
                 assert src[1] == pm.H2D and src[2] == 2 and (src[3], src[4]) == (i, j)
+
+
+def test_coherent_writebacks_in_completion_order():
+    """xk_memory_coherent_*: the D2H records of a view go out in the (virtual) completion order
+    of their tiles, so the FIFO D2H stream never waits behind a tile whose chain ends late."""
+    T, N = 4, 24
+    for G in (1, 4):
+        s = xk.PlanSession(uniform(G), topo="ranked", optimistic=True, tile=T)
+        recs = s.call(xk.make_call(m=N, n=N, k=N, alpha=1.5, beta=-0.75, A=A_ADDR, lda=N, B=B_ADDR, ldb=N,
+                                   C=C_ADDR, ldc=N, sync=False))
+        by_seq = {r[0]: r for r in recs}
+        wb = s.call(xk.make_call(routine=pm.COHERENT, m=N, n=N, C=C_ADDR, ldc=N))
+        s.close()
+        assert len(wb) == (N // T) ** 2 and all(r[1] == pm.D2H for r in wb)
+        done = [by_seq[r[14][0]][12] for r in wb]
+        assert done == sorted(done) and len(set(done)) > 1

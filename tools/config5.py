@@ -17,7 +17,8 @@ import paper_conf_sc_gautierl21_b200 as xk
 
 out = {"gpus": 1}
 N = int(os.environ.get("N5", 65536))
-tiles = [int(t) for t in os.environ.get("TILES", "2048,4096").split(",")]
+tiles = [int(t) for t in os.environ.get("TILES", "1024,2048,4096").split(",")]
+REPS = int(os.environ.get("REPS", 2))  # timed calls per tile, after one warm-up (paper: 8)
 A = inputs.uniform(1, N, N)
 B = inputs.uniform(2, N, N)
 C = inputs.uniform(3, N, N)
@@ -26,13 +27,20 @@ for T in tiles:
     xk.init(ngpus=1, tile=T, probe=True)
     for X in (A, B, C):
         xk.register(X)
-    torch.cuda.synchronize()
-    t0 = time.perf_counter()
-    xk.dgemm("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
-    torch.cuda.synchronize()
-    dt = time.perf_counter() - t0
+    xk.dgemm("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)  # warm-up (tile buffers allocated)
+    xk.reset_stats()
+    ts = []
+    for _ in range(REPS):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        xk.dgemm("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
+        torch.cuda.synchronize()
+        ts.append(time.perf_counter() - t0)
     st = xk.get_stats()
-    sweep[T] = {"tflops": 2.0 * N ** 3 / dt / 1e12, "s": dt, "h2d_GB": sum(st["h2d_bytes"]) / 1e9}
+    dt = sum(ts) / len(ts)
+    sweep[T] = {"tflops": 2.0 * N ** 3 / dt / 1e12, "s_mean": dt, "s_each": ts,
+                "h2d_GB_per_call": sum(st["h2d_bytes"]) / 1e9 / REPS, "timed_calls": REPS,
+                "tasks_per_call": sum(st["tasks"]) // REPS, "kernel_launches_per_call": st["kernel_launches"] // REPS}
     print("N=%d T=%d" % (N, T), sweep[T], flush=True)
     xk.finalize()
 out["dgemm_n%d_tile_sweep" % N] = sweep
