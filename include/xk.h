@@ -82,6 +82,25 @@ typedef struct xk_config {
     int kstreams;         /* kernel streams per GPU (0 = 2); plus 1 H2D, 1 D2H, 1 P2P-in */
     int probe;            /* 1 = time the (G+1)^2 link matrix at init (a1); 0 = defaults */
     int64_t task_rate_mflops; /* planner's tile-task rate (0 = derived from the FP64 peak) */
+    /* ---- rank mode: one process per GPU.  `world` processes each call
+     * xk_init with their own `rank` and the same `session`; process r drives logical GPU r
+     * only.  Every process runs the same deterministic planner on the same calls, so all
+     * hold the identical plan; each executes the records of its own GPU (H2D/P2P/task into
+     * it, D2H out of it), pulls peer tiles through CUDA IPC mappings of the peers' tile
+     * arenas and orders cross-process dependencies with per-record completion flags in the
+     * shared session file (stream memory operations, no host round trip).  In rank mode
+     * EVERY later API call is collective: all ranks make the same calls with the same
+     * arguments, host matrices live in memory shared by the processes (the same file
+     * mapping; addresses may differ per process), and xk_last_error() is per process.
+     * A failing rank marks the session so the others return XK_ERR_CUDA at their next
+     * synchronisation point instead of waiting forever. */
+    int rank;             /* this process's logical GPU, 0 <= rank < world */
+    int world;            /* number of processes = logical GPUs (0 or 1 = single-process mode) */
+    int64_t arena_bytes;  /* rank mode: device tile arena per GPU, the same on every rank
+                             (0 = 85% of the smallest free memory / ranks sharing a device) */
+    char session[128];    /* rank mode: path of the shared control file, unique per session
+                             (e.g. "/dev/shm/xk_<token>"); rank 0 creates it, rank 0 removes
+                             it at xk_finalize */
 } xk_config_t;
 
 /* Fill *cfg with defaults, then apply the environment (XK_NGPUS, XK_TILE,

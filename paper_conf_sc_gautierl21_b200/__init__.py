@@ -9,6 +9,7 @@ BLAS entry points return the BLAS info code (0, or -i for an invalid argument i)
 XKError for runtime failures (positive XK_ERR_* codes).
 """
 import ctypes
+import os
 
 from . import _abi
 from ._abi import (HOST, REC_D2H, REC_FIELDS, REC_H2D, REC_P2P, REC_TASK, ROUTINE_COHERENT,  # noqa: F401
@@ -57,8 +58,13 @@ def _c(ch):
 
 # ---------------------------------------------------------------------------- lifecycle
 def init(ngpus=0, tile=0, topo=None, optimistic=None, window=0, kstreams=0, probe=None,
-         grid=None, phys=None, task_rate_mflops=0):
-    """xk_init.  `phys` maps logical GPUs to physical devices (logical-device mode)."""
+         grid=None, phys=None, task_rate_mflops=0, rank=None, world=None, session=None, arena_bytes=0):
+    """xk_init.  `phys` maps logical GPUs to physical devices (logical-device mode).
+
+    Rank mode (one process per GPU): every one of `world` processes calls
+    init(rank=r, world=world, session=path) with the same unique `path` (see
+    new_session_path); from then on every call is collective and host matrices must live
+    in memory shared by the processes (shared_matrix)."""
     cfg = _abi.Config()
     lib().xk_config_default(ctypes.byref(cfg))
     if ngpus:
@@ -83,7 +89,34 @@ def init(ngpus=0, tile=0, topo=None, optimistic=None, window=0, kstreams=0, prob
             cfg.phys[i] = d
     if task_rate_mflops:
         cfg.task_rate_mflops = task_rate_mflops
+    if world is not None and world > 1:
+        cfg.rank, cfg.world = int(rank), int(world)
+        cfg.session = os.fsencode(session)
+        if phys is not None:  # phys[rank] = this process's device
+            cfg.map_devices = 1
+    if arena_bytes:
+        cfg.arena_bytes = int(arena_bytes)
     return _check(lib().xk_init(ctypes.byref(cfg)))
+
+
+# ---------------------------------------------------------------------------- rank mode
+def new_session_path(tag="xk"):
+    """A fresh path for the rank-mode session file (rank 0 picks it and shares it)."""
+    d = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
+    return os.path.join(d, "%s_%d_%s" % (tag, os.getpid(), os.urandom(6).hex()))
+
+
+def shared_matrix(path, rows, cols, create):
+    """A column-major float64 host matrix backed by a file mapping (MAP_SHARED) that every
+    rank-mode process maps: the "host memory" of the library's processes.  Plumbing only --
+    the creator sizes the file, the others open it; each process registers its own mapping."""
+    import numpy as np
+    nbytes = max(8, int(rows) * int(cols) * 8)
+    if create:
+        with open(path, "wb") as f:
+            f.truncate(nbytes)
+    mm = np.memmap(path, dtype=np.float64, mode="r+", shape=(int(rows), int(cols)), order="F")
+    return mm
 
 
 def finalize():

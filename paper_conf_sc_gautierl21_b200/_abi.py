@@ -37,7 +37,8 @@ class Config(ctypes.Structure):
     _fields_ = [("ngpus", c_int), ("phys", c_int * MAX_GPUS), ("map_devices", c_int),
                 ("grid_p", c_int), ("grid_q", c_int), ("tile", i64), ("topo", c_int),
                 ("optimistic", c_int), ("window", c_int), ("kstreams", c_int), ("probe", c_int),
-                ("task_rate_mflops", i64)]
+                ("task_rate_mflops", i64), ("rank", c_int), ("world", c_int), ("arena_bytes", i64),
+                ("session", ctypes.c_char * 128)]
 
 
 class Stats(ctypes.Structure):

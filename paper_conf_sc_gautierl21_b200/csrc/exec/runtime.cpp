@@ -12,6 +12,8 @@
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <chrono>
+#include <thread>
 
 #include "api/common.h"
 #include "kernels/kernels.h"
@@ -50,13 +52,24 @@ int Runtime::init(const xk_config_t &cfg) {
         set_error(std::string("no CUDA device: ") + cudaGetErrorString(e));
         return XK_ERR_NO_DEVICE;
     }
-    int G = cfg.ngpus > 0 ? cfg.ngpus : ndev;
+    rank_mode_ = cfg.world > 1;
+    if (rank_mode_ && (cfg.rank < 0 || cfg.rank >= cfg.world || (cfg.ngpus > 0 && cfg.ngpus != cfg.world))) {
+        set_error("config: rank mode needs 0 <= rank < world and ngpus in {0, world}");
+        return XK_ERR_CONFIG;
+    }
+    rank_ = rank_mode_ ? cfg.rank : 0;
+    int G = rank_mode_ ? cfg.world : cfg.ngpus > 0 ? cfg.ngpus : ndev;
     if (G > XK_MAX_GPUS) {
         set_error("ngpus > XK_MAX_GPUS");
         return XK_ERR_CONFIG;
     }
     devs_.assign(G, Device());
     for (int g = 0; g < G; ++g) {
+        if (rank_mode_ && g != rank_) {  // a peer process's GPU: no streams here
+            devs_[g].local = false;
+            devs_[g].phys = -1;
+            continue;
+        }
         int p = cfg.map_devices ? cfg.phys[g] : g % ndev;
         if (p < 0 || p >= ndev) {
             set_error("logical->physical device map out of range");
@@ -77,7 +90,7 @@ int Runtime::init(const xk_config_t &cfg) {
     for (int a = 0; a < G; ++a)
         for (int b = 0; b < G; ++b) {
             int pa = devs_[a].phys, pb = devs_[b].phys;
-            if (pa == pb) continue;
+            if (pa == pb || !devs_[a].local || !devs_[b].local) continue;
             int can = 0;
             XK_CK(cudaDeviceCanAccessPeer(&can, pa, pb));
             if (!can) continue;
@@ -88,6 +101,7 @@ int Runtime::init(const xk_config_t &cfg) {
         }
     for (int g = 0; g < G; ++g) {
         Device &d = devs_[g];
+        if (!d.local) continue;
         XK_CK(cudaSetDevice(d.phys));
         XK_CK(cudaStreamCreateWithFlags(&d.h2d, cudaStreamNonBlocking));
         XK_CK(cudaStreamCreateWithFlags(&d.d2h, cudaStreamNonBlocking));
@@ -120,6 +134,17 @@ int Runtime::init(const xk_config_t &cfg) {
         set_error("config: grid P*Q must equal ngpus; topo in {0,1,2}");
         return XK_ERR_CONFIG;
     }
+    if (rank_mode_) {
+        int rc = init_rank_mode(cfg);
+        if (rc) {
+            if (sess_) sess_->abort();
+            return rc;
+        }
+    }
+    // same physical device (logical-device mode, or ranks sharing a GPU)
+    auto same_dev = [&](int s, int d) {
+        return rank_mode_ ? devs_[s].pci == devs_[d].pci : devs_[s].phys == devs_[d].phys;
+    };
     // topology (a1): defaults, then the measured matrix when probing
     topo.G = G;
     topo.bw.assign((size_t)(G + 1) * (G + 1), 0);
@@ -128,7 +153,7 @@ int Runtime::init(const xk_config_t &cfg) {
             int64_t v;
             if (s == G || d == G) v = (s == d) ? 3000000 : 55000;
             else if (s == d) v = 3000000;
-            else v = (devs_[s].phys == devs_[d].phys) ? 1500000 : 700000;
+            else v = same_dev(s, d) ? 1500000 : 700000;
             topo.bw[(size_t)s * (G + 1) + d] = v;
         }
     topo.rate_mflops = cfg.task_rate_mflops > 0 ? cfg.task_rate_mflops : 35000000;
@@ -136,15 +161,18 @@ int Runtime::init(const xk_config_t &cfg) {
     for (int s = 0; s < G; ++s)
         for (int d = 0; d < G; ++d) {
             int ps = devs_[s].phys, pd = devs_[d].phys;
-            if (ps == pd) continue;
+            if (ps == pd || !devs_[s].local || !devs_[d].local) continue;
             int v = 0;
             if (cudaDeviceGetP2PAttribute(&v, cudaDevP2PAttrPerformanceRank, ps, pd) == cudaSuccess)
                 perf_rank[(size_t)s * G + d] = v;
             cudaGetLastError();
         }
     if (cfg.probe) {
-        int rc = probe_topology();
-        if (rc) return rc;
+        int rc = rank_mode_ ? probe_topology_rank() : probe_topology();
+        if (rc) {
+            if (sess_) sess_->abort();
+            return rc;
+        }
     }
     planner_.reset(new Planner(topo, flags_));
     std::memset(&stats, 0, sizeof(stats));
@@ -242,6 +270,173 @@ int Runtime::probe_topology() {
     return XK_OK;
 }
 
+// Rank mode set-up: open the session file, map its flag array into this
+// GPU's address space, agree on one arena size, allocate this GPU's tile arena and map
+// every peer's arena through CUDA IPC.  Collective: every rank runs it in xk_init.
+int Runtime::init_rank_mode(const xk_config_t &cfg) {
+    const int G = (int)devs_.size();
+    if (!stream_memops_available()) {
+        set_error("rank mode: cuStreamWaitValue32/cuStreamWriteValue32 unavailable");
+        return XK_ERR_CUDA;
+    }
+    std::string path(cfg.session, strnlen(cfg.session, sizeof cfg.session));
+    if (path.empty()) {
+        set_error("config: rank mode needs xk_config_t.session (a unique file path)");
+        return XK_ERR_CONFIG;
+    }
+    sess_.reset(new Session());
+    std::string err;
+    int rc = sess_->open(path, rank_, G, 300.0, err);
+    if (rc) {
+        set_error(err);
+        sess_.reset();
+        return rc;
+    }
+    SessionHeader *h = sess_->hdr();
+    SessionRank &me = h->rank[rank_];
+    Device &d = devs_[rank_];
+    XK_CK(cudaSetDevice(d.phys));
+    XK_CK(cudaHostRegister(sess_->flags(), sess_->flags_bytes(), cudaHostRegisterPortable | cudaHostRegisterMapped));
+    XK_CK(cudaHostGetDevicePointer((void **)&dflags_, sess_->flags(), 0));
+    int dom = 0, bus = 0, dv = 0;
+    XK_CK(cudaDeviceGetAttribute(&dom, cudaDevAttrPciDomainId, d.phys));
+    XK_CK(cudaDeviceGetAttribute(&bus, cudaDevAttrPciBusId, d.phys));
+    XK_CK(cudaDeviceGetAttribute(&dv, cudaDevAttrPciDeviceId, d.phys));
+    me.pci = (dom << 16) | (bus << 8) | dv;
+    auto bar = [&](const char *what) {
+        if (sess_->barrier(300.0)) return XK_OK;
+        set_error(std::string("rank mode: a peer failed or timed out during ") + what);
+        return XK_ERR_CUDA;
+    };
+    if ((rc = bar("init (device ids)"))) return rc;
+    int share = 0;
+    for (int g = 0; g < G; ++g) {
+        devs_[g].pci = h->rank[g].pci;
+        share += h->rank[g].pci == me.pci;
+    }
+    size_t fr = 0, tot = 0;
+    XK_CK(cudaMemGetInfo(&fr, &tot));
+    me.arena_proposed = cfg.arena_bytes > 0 ? cfg.arena_bytes : (int64_t)((double)fr * 0.85) / std::max(1, share);
+    if ((rc = bar("init (arena size)"))) return rc;
+    int64_t ab = h->rank[0].arena_proposed;
+    for (int g = 1; g < G; ++g) ab = std::min(ab, h->rank[g].arena_proposed);
+    ab = ab / (2 << 20) * (2 << 20);
+    if (ab < ((int64_t)256 << 20)) {
+        set_error("rank mode: arena smaller than 256 MiB");
+        return XK_ERR_OOM;
+    }
+    void *arena = nullptr;
+    cudaError_t e = cudaMalloc(&arena, (size_t)ab);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error("rank mode: cannot allocate the device tile arena");
+        return XK_ERR_OOM;
+    }
+    d.arena = static_cast<char *>(arena);
+    d.arena_bytes = ab;
+    XK_CK(cudaIpcGetMemHandle(&me.arena, arena));
+    me.arena_bytes = ab;
+    if ((rc = bar("init (arena handles)"))) return rc;
+    for (int g = 0; g < G; ++g) {
+        if (g == rank_) continue;
+        void *p = nullptr;
+        XK_CK(cudaIpcOpenMemHandle(&p, h->rank[g].arena, cudaIpcMemLazyEnablePeerAccess));
+        devs_[g].arena = static_cast<char *>(p);
+        devs_[g].arena_bytes = h->rank[g].arena_bytes;
+    }
+    cur_dev_ = -1;
+    return bar("init (arena mappings)");
+}
+
+// a1 in rank mode: each process times its own host links and local copies, then pulls
+// 64 MiB from every peer's arena in G-1 barrier-separated rounds (round j: rank r pulls
+// from rank r-j, a permutation, so no two pulls share a source); the rows meet in the
+// session file and every process builds the identical matrix the planner needs.
+int Runtime::probe_topology_rank() {
+    const int G = (int)devs_.size(), N = G + 1;
+    const size_t bytes = (size_t)64 << 20;
+    Device &d = devs_[rank_];
+    SessionHeader *h = sess_->hdr();
+    SessionRank &me = h->rank[rank_];
+    int rc;
+    if ((rc = set_dev(rank_))) return rc;
+    void *host = nullptr;
+    XK_CK(cudaMallocHost(&host, bytes));
+    std::memset(host, 1, bytes);
+    char *src0 = d.arena, *dst = d.arena + bytes;
+    auto timed = [&](cudaStream_t s, auto fn, float *ms_out) -> int {
+        cudaEvent_t a, b;
+        XK_CK(cudaEventCreate(&a));
+        XK_CK(cudaEventCreate(&b));
+        float best = 1e30f;
+        for (int rep = 0; rep < 3; ++rep) {
+            XK_CK(cudaEventRecord(a, s));
+            XK_CK(fn());
+            XK_CK(cudaEventRecord(b, s));
+            XK_CK(cudaEventSynchronize(b));
+            float ms = 0;
+            XK_CK(cudaEventElapsedTime(&ms, a, b));
+            if (rep > 0) best = std::min(best, ms);
+        }
+        cudaEventDestroy(a);
+        cudaEventDestroy(b);
+        *ms_out = best;
+        return XK_OK;
+    };
+    auto mbps = [&](float ms) { return (int64_t)((double)bytes / (ms * 1e-3) / 1e6); };
+    float ms;
+    if ((rc = timed(d.h2d, [&] { return cudaMemcpyAsync(src0, host, bytes, cudaMemcpyHostToDevice, d.h2d); }, &ms))) return rc;
+    me.bw_in[G] = mbps(ms);
+    if ((rc = timed(d.d2h, [&] { return cudaMemcpyAsync(host, src0, bytes, cudaMemcpyDeviceToHost, d.d2h); }, &ms))) return rc;
+    me.bw_to_host = mbps(ms);
+    if ((rc = timed(d.p2p, [&] { return cudaMemcpyAsync(dst, src0, bytes, cudaMemcpyDeviceToDevice, d.p2p); }, &ms))) return rc;
+    me.bw_local = mbps(ms);
+    cudaFreeHost(host);
+    for (int j = 1; j < G; ++j) {
+        if (!sess_->barrier(300.0)) {
+            set_error("rank mode: a peer failed during the topology probe");
+            return XK_ERR_CUDA;
+        }
+        const int s = (rank_ - j + G) % G;
+        const char *src = devs_[s].arena;
+        if ((rc = timed(d.p2p, [&] { return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToDevice, d.p2p); }, &ms))) return rc;
+        me.bw_in[s] = mbps(ms);
+    }
+    // FP64 tile-task rate, measured by rank 0 for everyone (T <= 2048, in its arena)
+    me.rate_mflops = 0;
+    if (rank_ == 0 && cfg_.task_rate_mflops <= 0) {
+        const int64_t T = std::min<int64_t>(flags_.T, 2048);
+        const size_t tb = (size_t)T * T * 8;
+        if ((int64_t)(3 * tb) <= d.arena_bytes) {
+            double *a = reinterpret_cast<double *>(d.arena), *b = a + (size_t)T * T, *c = b + (size_t)T * T;
+            XK_CK(cudaMemsetAsync(d.arena, 0, 3 * tb, d.ks[0]));
+            if ((rc = timed(d.ks[0], [&] { return launch_dgemm_tile(false, false, T, T, T, 1.0, a, T, b, T, 1.0, c, T, d.ks[0]); }, &ms))) return rc;
+            me.rate_mflops = std::max<int64_t>(1, (int64_t)(2.0 * T * T * T / (ms * 1e3)));
+        }
+    }
+    if (!sess_->barrier(300.0)) {
+        set_error("rank mode: a peer failed during the topology probe");
+        return XK_ERR_CUDA;
+    }
+    for (int g = 0; g < G; ++g) {
+        const SessionRank &sr = h->rank[g];
+        for (int s = 0; s < G; ++s)
+            if (s != g) topo.bw[(size_t)s * N + g] = sr.bw_in[s];
+        topo.bw[(size_t)G * N + g] = sr.bw_in[G];
+        topo.bw[(size_t)g * N + G] = sr.bw_to_host;
+        topo.bw[(size_t)g * N + g] = sr.bw_local;
+    }
+    topo.bw[(size_t)G * N + G] = topo.bw[0];
+    if (cfg_.task_rate_mflops <= 0 && h->rank[0].rate_mflops > 0) topo.rate_mflops = h->rank[0].rate_mflops;
+    cur_dev_ = -1;
+    // nobody reuses its arena (tile allocations start at offset 0) before every pull is done
+    if (!sess_->barrier(300.0)) {
+        set_error("rank mode: a peer failed during the topology probe");
+        return XK_ERR_CUDA;
+    }
+    return XK_OK;
+}
+
 cudaEvent_t Runtime::new_event(int g) {
     auto &pool = ev_pool_[g];
     cudaEvent_t e = nullptr;
@@ -265,6 +460,11 @@ int Runtime::record(cudaStream_t s, int g, Ev *out) {
 }
 
 int Runtime::wait_on(cudaStream_t s, const Ev &ev) {
+    if (ev.rseq >= 0) {  // executed by a peer process: its completion flag
+        if (ev.rseq < epoch_seq_) return XK_OK;
+        XK_CK(stream_wait_flag(s, dflags_ + (uint64_t)ev.rseq % kFlagCap, (uint32_t)(ev.rseq + 1)));
+        return XK_OK;
+    }
     if (!ev.e || ev.s == s) return XK_OK;  // same stream: already ordered
     XK_CK(cudaStreamWaitEvent(s, ev.e, 0));
     return XK_OK;
@@ -273,13 +473,22 @@ int Runtime::wait_on(cudaStream_t s, const Ev &ev) {
 int Runtime::wait_dep(cudaStream_t s, int64_t seq) {
     if (seq < 0) return XK_OK;
     auto it = seq_ev_.find(seq);
-    if (it == seq_ev_.end()) return XK_OK;  // completed before the last full sync
-    return wait_on(s, it->second);
+    if (it != seq_ev_.end()) return wait_on(s, it->second);
+    // not issued here since the last full sync: completed before it, or (rank mode)
+    // executed by a peer process -- local records are always issued before a dependant
+    if (rank_mode_ && seq >= epoch_seq_) return wait_on(s, Ev::remote(seq));
+    return XK_OK;
+}
+
+int Runtime::signal(cudaStream_t s, int64_t seq) {
+    if (!rank_mode_) return XK_OK;
+    XK_CK(stream_write_flag(s, dflags_ + (uint64_t)seq % kFlagCap, (uint32_t)(seq + 1)));
+    return XK_OK;
 }
 
 static void add_reader(Buffer &b, const Ev &ev) {
     for (auto &r : b.readers)
-        if (r.s == ev.s) {  // in-order stream: the newer event subsumes the older one
+        if (ev.rseq < 0 && r.rseq < 0 && r.s == ev.s) {  // in-order stream: the newer event subsumes the older one
             r = ev;
             return;
         }
@@ -294,6 +503,19 @@ double *Runtime::alloc(int g, size_t bytes, int *rc) {
         it->second.pop_back();
         d.bytes_in_use += bytes;
         return p;
+    }
+    if (rank_mode_) {
+        // every process runs this allocator for EVERY GPU in plan order, so all agree on
+        // where each tile lives in each arena without exchanging a message
+        const int64_t off = round_up(d.arena_top, 1024);
+        if (off + (int64_t)bytes > d.arena_bytes) {
+            set_error("rank mode: device tile arena full (no eviction): raise xk_config_t.arena_bytes");
+            *rc = XK_ERR_OOM;
+            return nullptr;
+        }
+        d.arena_top = off + (int64_t)bytes;
+        d.bytes_in_use += bytes;
+        return reinterpret_cast<double *>(d.arena + off);
     }
     if ((*rc = set_dev(g))) return nullptr;
     double *p = nullptr;
@@ -358,7 +580,11 @@ int Runtime::issue(const Rec &R) {
     // the D2H of a tile whose last writer is still in this GPU's pending batch waits for the
     // batch instead of launching it early (a step's diagonal ops / GEMMs stay one launch) --
     // except in the GPU's last tasks of the call, where the write-back is the tail
-    if (defer_d2h_ && r.kind == XK_REC_D2H && r.dep[0] >= 0 && batch_[r.src].contains_seq(r.dep[0]) &&
+    if (rank_mode_ && r.seq - epoch_seq_ >= (int64_t)(kFlagCap / 2)) {
+        set_error("rank mode: more plan records in flight than the completion-flag ring holds");
+        return XK_ERR_UNSUPPORTED;
+    }
+    if (defer_d2h_ && here(r) && r.kind == XK_REC_D2H && r.dep[0] >= 0 && batch_[r.src].contains_seq(r.dep[0]) &&
         batch_[r.src].recs.back().remaining >= max_batch_) {
         PendingBatch &bt = batch_[r.src];
         bt.deferred.push_back(R);
@@ -367,6 +593,7 @@ int Runtime::issue(const Rec &R) {
         return XK_OK;
     }
     if (r.kind != XK_REC_TASK && (rc = flush_for(R))) return rc;
+    if (!here(r)) return issue_remote(R);
     switch (r.kind) {
     case XK_REC_H2D: {
         const int g = r.dst;
@@ -385,6 +612,7 @@ int Runtime::issue(const Rec &R) {
         if (tracing_) trace_end(g, s, ta, 0, "H2D", r.work);
         Ev ev;
         if ((rc = record(s, g, &ev))) return rc;
+        if ((rc = signal(s, r.seq))) return rc;
         seq_ev_[r.seq] = ev;
         B->writer = ev;
         B->readers.clear();
@@ -413,6 +641,7 @@ int Runtime::issue(const Rec &R) {
         if (tracing_) trace_end(g, s, ta, 1, r.src_state == XK_SRC_INFLIGHT ? "P2P fwd-inflight" : "P2P", r.work);
         Ev ev;
         if ((rc = record(s, g, &ev))) return rc;
+        if ((rc = signal(s, r.seq))) return rc;
         seq_ev_[r.seq] = ev;
         D->writer = ev;
         D->readers.clear();
@@ -499,6 +728,7 @@ int Runtime::issue(const Rec &R) {
             }
             Ev ev;
             if ((rc = record(s, g, &ev))) return rc;
+            if ((rc = signal(s, r.seq))) return rc;
             seq_ev_[r.seq] = ev;
             O->writer = ev;
             O->readers.clear();
@@ -558,6 +788,7 @@ int Runtime::issue(const Rec &R) {
         if (tracing_) trace_end(gs, s, ta, 3, "D2H", r.work);
         Ev ev;
         if ((rc = record(s, gs, &ev))) return rc;
+        if ((rc = signal(s, r.seq))) return rc;
         seq_ev_[r.seq] = ev;
         add_reader(*S, ev);
         pending_d2h_.push_back(ev);
@@ -565,6 +796,50 @@ int Runtime::issue(const Rec &R) {
         stats.link_bytes[(size_t)gs * (devs_.size() + 1) + devs_.size()] += r.work;
         return XK_OK;
     }
+    default:
+        set_error("internal: unknown record kind");
+        return XK_ERR_INTERNAL;
+    }
+}
+
+// Rank mode: a record another process executes.  Nothing is enqueued here; the directory
+// of buffers is kept identical on every process (same allocations, in plan order), the
+// peer's output is known only by its completion flag, and a P2P that pulls one of OUR
+// tiles becomes a remote reader of it (a later overwrite waits for the pull's flag).
+int Runtime::issue_remote(const Rec &R) {
+    const xk_plan_rec_t &r = R.r;
+    int rc = XK_OK;
+    switch (r.kind) {
+    case XK_REC_H2D:
+    case XK_REC_P2P: {
+        Buffer *D = buf(R.key, r.dst, true, &rc);
+        if (!D) return rc;
+        D->writer = Ev::remote(r.seq);
+        D->readers.clear();
+        if (r.kind == XK_REC_P2P && r.src == rank_) {
+            Buffer *S = buf(R.key, r.src, false, &rc);
+            if (!S) return rc;
+            add_reader(*S, Ev::remote(r.seq));
+            stats.p2p_out_bytes[rank_] += r.work;  // pulled by the peer, counted at the source too
+        }
+        return XK_OK;
+    }
+    case XK_REC_TASK: {
+        Buffer *O = buf(R.key, r.dst, true, &rc);
+        if (!O) return rc;
+        O->writer = Ev::remote(r.seq);
+        O->readers.clear();
+        if (R.op == XK_OP_SYMM_DIAG) {  // the owner's scratch tile, same size and order
+            const int64_t ka = (R.side == 'L') ? R.m : R.n;
+            const size_t sb = (size_t)((ka + 15) / 16 * 16) * ka * 8;
+            double *S = alloc(r.dst, sb, &rc);
+            if (!S) return rc;
+            scratch_.push_back({r.dst, {S, sb}});
+        }
+        return XK_OK;
+    }
+    case XK_REC_D2H:
+        return XK_OK;
     default:
         set_error("internal: unknown record kind");
         return XK_ERR_INTERNAL;
@@ -620,6 +895,7 @@ int Runtime::flush_batch(int g) {
         if ((rc = record(s, g, &ev))) return rc;
         for (int q = 0; q < nb; ++q) {
             const Rec &R = bt.recs[q];
+            if ((rc = signal(s, R.r.seq))) return rc;
             seq_ev_[R.r.seq] = ev;
             Buffer *O = buf(R.key, g, false, &rc);
             O->writer = ev;
@@ -674,6 +950,7 @@ int Runtime::flush_batch(int g) {
     if ((rc = record(s, g, &ev))) return rc;
     for (int q = 0; q < tb.n; ++q) {
         const Rec &R = bt.recs[q];
+        if ((rc = signal(s, R.r.seq))) return rc;
         seq_ev_[R.r.seq] = ev;
         Buffer *O = buf(R.key, g, false, &rc);
         O->writer = ev;
@@ -773,6 +1050,7 @@ int Runtime::trace_start(const std::string &path) {
     trace_json_.clear();
     trace_base_.assign(devs_.size(), nullptr);
     for (size_t g = 0; g < devs_.size(); ++g) {
+        if (!devs_[g].local) continue;
         XK_CK(cudaSetDevice(devs_[g].phys));
         XK_CK(cudaEventCreate(&trace_base_[g]));
         XK_CK(cudaEventRecord(trace_base_[g], devs_[g].h2d));
@@ -945,28 +1223,77 @@ int Runtime::unregister_host(void *p) {
 }
 
 void Runtime::release_invalid() {
-    for (auto it = bufs_.begin(); it != bufs_.end();) {
-        int key = (int)(it->first / XK_MAX_GPUS), g = (int)(it->first % XK_MAX_GPUS);
-        if (!planner_->entry(key).gpu[g].present) {
-            free_buf(g, it->second.p, it->second.bytes);
-            it = bufs_.erase(it);
-        } else {
-            ++it;
+    // in id order: the free lists (and so every later placement) come out the same in
+    // every process of rank mode
+    std::vector<int64_t> ids;
+    for (auto &kv : bufs_) {
+        int key = (int)(kv.first / XK_MAX_GPUS), g = (int)(kv.first % XK_MAX_GPUS);
+        if (!planner_->entry(key).gpu[g].present) ids.push_back(kv.first);
+    }
+    std::sort(ids.begin(), ids.end());
+    for (int64_t id : ids) {
+        Buffer &b = bufs_[id];
+        free_buf((int)(id % XK_MAX_GPUS), b.p, b.bytes);
+        bufs_.erase(id);
+    }
+}
+
+int Runtime::wait_stream(cudaStream_t s) {
+    if (!rank_mode_) {
+        XK_CK(cudaStreamSynchronize(s));
+        return XK_OK;
+    }
+    // a stream may wait on a peer's completion flag: never block without watching the
+    // session's abort flag
+    for (int spins = 0;; ++spins) {
+        cudaError_t e = cudaStreamQuery(s);
+        if (e == cudaSuccess) return XK_OK;
+        if (e != cudaErrorNotReady) return cuda_fail(e, "cudaStreamQuery");
+        if (sess_->aborted()) {
+            set_error("rank mode: a peer process failed");
+            return XK_ERR_CUDA;
         }
+        if (spins > 200) std::this_thread::sleep_for(std::chrono::microseconds(20));
+    }
+}
+
+int Runtime::wait_event(cudaEvent_t ev) {
+    if (!rank_mode_) {
+        XK_CK(cudaEventSynchronize(ev));
+        return XK_OK;
+    }
+    for (int spins = 0;; ++spins) {
+        cudaError_t e = cudaEventQuery(ev);
+        if (e == cudaSuccess) return XK_OK;
+        if (e != cudaErrorNotReady) return cuda_fail(e, "cudaEventQuery");
+        if (sess_->aborted()) {
+            set_error("rank mode: a peer process failed");
+            return XK_ERR_CUDA;
+        }
+        if (spins > 200) std::this_thread::sleep_for(std::chrono::microseconds(20));
     }
 }
 
 int Runtime::sync_all() {
+    int rc;
     for (size_t g = 0; g < devs_.size(); ++g) {
         Device &d = devs_[g];
+        if (!d.local) continue;
         XK_CK(cudaSetDevice(d.phys));
-        XK_CK(cudaStreamSynchronize(d.h2d));
-        XK_CK(cudaStreamSynchronize(d.p2p));
-        for (int k = 0; k < nks_; ++k) XK_CK(cudaStreamSynchronize(d.ks[k]));
-        XK_CK(cudaStreamSynchronize(d.kdiag));
-        XK_CK(cudaStreamSynchronize(d.d2h));
+        if ((rc = wait_stream(d.h2d)) || (rc = wait_stream(d.p2p))) return rc;
+        for (int k = 0; k < nks_; ++k)
+            if ((rc = wait_stream(d.ks[k]))) return rc;
+        if ((rc = wait_stream(d.kdiag)) || (rc = wait_stream(d.d2h))) return rc;
     }
     cur_dev_ = -1;
+    if (rank_mode_) {
+        // every process's streams are idle: every record planned so far has completed
+        if (!sess_->barrier()) {
+            set_error("rank mode: a peer process failed or timed out at a synchronisation point");
+            return XK_ERR_CUDA;
+        }
+        if (planner_) epoch_seq_ = planner_->next_seq();
+    }
     if (tracing_) trace_collect();
     for (size_t q = 0; q < ktimers_.size(); ++q) {
         float ms = 0;
@@ -988,6 +1315,7 @@ int Runtime::sync_all() {
         kv.second.readers.clear();
     }
     for (size_t g = 0; g < devs_.size(); ++g) {
+        if (!devs_[g].local) continue;
         for (cudaEvent_t e : ev_used_[g]) ev_pool_[g].push_back(e);
         ev_used_[g].clear();
     }
@@ -1004,7 +1332,13 @@ int Runtime::run(const xk_call_t &call, bool wait) {
         return failed_;
     }
     cur_dev_ = -1;
-    int rc = run_impl(call, wait);
+    int rc = XK_OK;
+    // rank mode: keep the records in flight well inside the completion-flag ring (every
+    // process takes this branch at the same call: the plans are identical)
+    if (rank_mode_ && call.routine != XK_ROUTINE_SYNC && planner_->next_seq() - epoch_seq_ > (int64_t)(kFlagCap / 4))
+        rc = sync_all();
+    if (!rc) rc = run_impl(call, wait);
+    if (rc && rank_mode_ && sess_) sess_->abort();
     // after a runtime failure mid-call the directory may describe copies that were never
     // made: refuse further work until re-initialisation (never compute on a stale cache)
     if (rc == XK_ERR_CUDA || rc == XK_ERR_OOM || rc == XK_ERR_INTERNAL) failed_ = rc;
@@ -1079,7 +1413,13 @@ int Runtime::run_impl(const xk_call_t &call, bool wait) {
         return XK_OK;
     }
     if (wait) {
-        for (size_t q = d2h0; q < pending_d2h_.size(); ++q) XK_CK(cudaEventSynchronize(pending_d2h_[q].e));
+        for (size_t q = d2h0; q < pending_d2h_.size(); ++q)
+            if ((rc = wait_event(pending_d2h_[q].e))) return rc;
+        // rank mode: the host view is coherent once every process's write-backs landed
+        if (rank_mode_ && !sess_->barrier()) {
+            set_error("rank mode: a peer process failed or timed out at a synchronisation point");
+            return XK_ERR_CUDA;
+        }
     }
     return XK_OK;
 }
@@ -1101,10 +1441,20 @@ int Runtime::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
 int Runtime::finalize() {
     std::lock_guard<std::recursive_mutex> lk(mu);
     if (tracing_) trace_stop();
-    int rc = sync_all();
+    const bool peer_failed = rank_mode_ && sess_ && sess_->aborted();
+    int rc = peer_failed ? XK_ERR_CUDA : sync_all();
+    if (rank_mode_) {
+        // close the mappings of the peers' arenas before anyone frees its own
+        for (Device &d : devs_)
+            if (!d.local && d.arena) cudaIpcCloseMemHandle(d.arena);
+        if (sess_ && !peer_failed) sess_->barrier(120.0);
+    }
     for (size_t g = 0; g < devs_.size(); ++g) {
         Device &d = devs_[g];
+        if (!d.local) continue;
         cudaSetDevice(d.phys);
+        if (rank_mode_ && d.arena) cudaFree(d.arena);
+        d.arena = nullptr;
         for (auto &pb : d.all_bufs) cudaFree(pb.first);
         d.all_bufs.clear();
         d.free_bufs.clear();
@@ -1119,6 +1469,12 @@ int Runtime::finalize() {
     release_internal_pins();
     for (auto &kv : registered_) cudaHostUnregister((void *)kv.first);
     registered_.clear();
+    if (sess_) {
+        if (sess_->flags()) cudaHostUnregister(sess_->flags());
+        cudaGetLastError();
+        sess_->close(rank_ == 0);
+        sess_.reset();
+    }
     planner_.reset();
     devs_.clear();
     return rc;

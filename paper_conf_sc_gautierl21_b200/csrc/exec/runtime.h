@@ -15,6 +15,7 @@
 #include <vector>
 
 #include "kernels/kernels.h"
+#include "exec/session.h"
 #include "plan/plan.h"
 #include "xk.h"
 
@@ -25,6 +26,8 @@ constexpr int kMaxKStreams = 8;
 struct Ev {
     cudaEvent_t e = nullptr;
     cudaStream_t s = nullptr;  // stream it was recorded on
+    int64_t rseq = -1;         // rank mode: plan record executed by another process (flag wait)
+    static Ev remote(int64_t seq) { Ev v; v.rseq = seq; return v; }
 };
 
 // A device tile: compact column-major, ld = rows rounded up to 16 (128-byte columns).
@@ -62,6 +65,10 @@ struct PendingBatch {
 
 struct Device {
     int phys = 0;
+    bool local = true;    // rank mode: only the process's own GPU has streams
+    int pci = 0;          // PCI id of the physical device (rank mode: from the session)
+    char *arena = nullptr;       // rank mode: device tile arena (own: cudaMalloc; peer: IPC mapping)
+    int64_t arena_bytes = 0, arena_top = 0;
     cudaStream_t h2d = nullptr, d2h = nullptr, p2p = nullptr;
     cudaStream_t ks[kMaxKStreams] = {};
     cudaStream_t kdiag = nullptr;  // highest priority: diagonal-tile ops (critical path of TRSM)
@@ -119,6 +126,21 @@ private:
     int copy_host(bool h2d, double *dev, int64_t dld, char *host, int64_t hld, int64_t rows,
                   int64_t cols, cudaStream_t s);
     int set_dev(int g);
+    // ---- rank mode (one process per GPU)
+    bool here(const xk_plan_rec_t &r) const {
+        return !rank_mode_ || (r.kind == XK_REC_D2H ? r.src : r.dst) == rank_;
+    }
+    int init_rank_mode(const xk_config_t &cfg);
+    int probe_topology_rank();
+    int signal(cudaStream_t s, int64_t seq);   // completion flag of a locally executed record
+    int wait_stream(cudaStream_t s);           // abort-aware stream synchronisation
+    int wait_event(cudaEvent_t e);
+    int issue_remote(const Rec &R);
+    bool rank_mode_ = false;
+    int rank_ = 0;
+    std::unique_ptr<Session> sess_;
+    uint32_t *dflags_ = nullptr;  // device address of the session's flag array
+    int64_t epoch_seq_ = 0;       // records below this completed at the last full sync
 
     xk_config_t cfg_{};
     Flags flags_;

@@ -100,6 +100,7 @@ public:
         return (int)((i % flags_.P) * flags_.Q + (j % flags_.Q));
     }
     const Flags &flags() const { return flags_; }
+    int64_t next_seq() const { return seq_; }  // seq of the next record to be emitted
     int link_class(int s, int d) const { return cls_[(size_t)s * (topo_.G + 1) + d]; }
 
 private:

@@ -1,0 +1,130 @@
+"""Rank mode -- one process per GPU -- through the C ABI.
+
+`world` processes (tests/rank_worker.py) share a session file and host matrices in shared
+file mappings.  Each runs the same deterministic planner and executes only its own GPU's
+records: peer tiles are pulled through CUDA IPC mappings of the other processes' arenas,
+cross-process dependencies are per-record completion flags (stream memory operations).
+On a one-GPU box every rank maps to the same device (the IPC pulls are then device-local
+copies); on a multi-GPU box rank r runs on GPU r.
+
+Checks: exact-integer results bitwise equal to the CPU oracle (TRSM: Q13 residual bound +
+relative Frobenius); every rank's measured H2D / P2P-in / D2H bytes equal the bytes the
+plan assigns to its GPU (the planner replayed on the CPU with the same topology); closed
+forms for the composed call (D never crosses PCIe).
+"""
+import json
+import os
+import subprocess
+import sys
+import tempfile
+
+import pytest
+
+import paper_conf_sc_gautierl21_b200 as xk
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def run_ranks(world, case, n=1000, tile=256, probe=0, timeout=600):
+    with tempfile.TemporaryDirectory(dir="/dev/shm" if os.path.isdir("/dev/shm") else None) as d:
+        session = os.path.join(d, "session")
+        procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "rank_worker.py"),
+                                   "--rank", str(r), "--world", str(world), "--session", session,
+                                   "--dir", d, "--case", case, "--n", str(n), "--tile", str(tile),
+                                   "--probe", str(probe), "--arena", str(1 << 30)],
+                                  stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True, cwd=ROOT)
+                 for r in range(world)]
+        outs = []
+        try:
+            for p in procs:
+                o, e = p.communicate(timeout=timeout)
+                assert p.returncode == 0, e[-3000:]
+                outs.append(json.loads(o.strip().splitlines()[-1]))
+        finally:
+            for p in procs:
+                if p.poll() is None:
+                    p.kill()
+        assert not os.path.exists(session), "rank 0 removes the session file at finalize"
+    outs.sort(key=lambda o: o["rank"])
+    assert outs[0]["ok"], outs[0].get("failed")
+    return outs
+
+
+def plan_bytes(topo, calls, tile, world):
+    """Per-GPU H2D / P2P-in / D2H bytes of the plan, replayed on the CPU planner."""
+    s = xk.PlanSession(topo["bw_MBps"], topo["task_rate_mflops"], tile=tile)
+    h2d, p2p, d2h = [0] * world, [0] * world, [0] * world
+    try:
+        for c in calls:
+            for rec in s.call(c, cap=1 << 18):
+                r = dict(zip(xk.REC_FIELDS, rec))
+                if r["kind"] == xk.REC_H2D:
+                    h2d[r["dst"]] += r["work"]
+                elif r["kind"] == xk.REC_P2P:
+                    p2p[r["dst"]] += r["work"]
+                elif r["kind"] == xk.REC_D2H:
+                    d2h[r["src"]] += r["work"]
+    finally:
+        s.close()
+    return h2d, p2p, d2h
+
+
+def assert_bytes_follow_plan(outs, calls, tile):
+    world = len(outs)
+    topo = outs[0]["topology"]
+    for o in outs[1:]:
+        assert o["topology"] == topo, "every rank must build the identical link matrix"
+    h2d, p2p, d2h = plan_bytes(topo, calls, tile, world)
+    for o in outs:
+        r, st = o["rank"], o["stats"]
+        assert (st["h2d_bytes"], st["p2p_in_bytes"], st["d2h_bytes"]) == (h2d[r], p2p[r], d2h[r]), (r, st)
+    assert sum(o["stats"]["p2p_in_bytes"] for o in outs) == sum(o["stats"]["p2p_out_bytes"] for o in outs)
+
+
+BASE = 1 << 40  # fake, non-overlapping host addresses for the CPU replay of the calls
+
+
+def addr(i, n):
+    return BASE + i * (8 * n * n + (1 << 20))
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_rank_mode_gemm_bitwise_and_bytes(world):
+    N, T = 1000, 256
+    outs = run_ranks(world, "gemm", N, T)
+    A, B, C, E = (addr(i, N) for i in range(4))
+    calls = [xk.make_call(m=N, n=N, k=N, alpha=-2.0, beta=0.5, A=A, lda=N, B=B, ldb=N, C=C, ldc=N, sync=True),
+             xk.make_call(transA="T", m=N, n=N, k=N, alpha=1.0, beta=0.0, A=A, lda=N, B=C, ldb=N, C=E, ldc=N,
+                          sync=True)]
+    assert_bytes_follow_plan(outs, calls, T)
+    assert sum(o["stats"]["p2p_in_bytes"] for o in outs) > 0, "tiles must be forwarded between processes"
+
+
+def test_rank_mode_composition_no_h2d_of_intermediate():
+    world, N, T = 4, 1000, 256
+    outs = run_ranks(world, "compose", N, T)
+    A, B, C, E, D = (addr(i, N) for i in range(5))
+    calls = [xk.make_call(m=N, n=N, k=N, alpha=1.0, beta=0.0, A=A, lda=N, B=B, ldb=N, C=D, ldc=N),
+             xk.make_call(m=N, n=N, k=N, alpha=1.0, beta=0.0, A=D, lda=N, B=C, ldb=N, C=E, ldc=N),
+             xk.make_call(routine=xk.ROUTINE_COHERENT, m=N, n=N, C=E, ldc=N),
+             xk.make_call(routine=xk.ROUTINE_COHERENT, m=N, n=N, C=D, ldc=N)]
+    assert_bytes_follow_plan(outs, calls, T)
+    h2d = sum(o["stats"]["h2d_bytes"] for o in outs)
+    d2h = sum(o["stats"]["d2h_bytes"] for o in outs)
+    assert h2d == 3 * 8 * N * N, "A, B, C each cross PCIe once; D never does"
+    assert d2h == 2 * 8 * N * N
+
+
+def test_rank_mode_data_on_device_and_probe():
+    """Prefetched operands (data-on-device): the GEMM moves no host bytes; the link matrix
+    is probed collectively (every rank must end with the same matrix)."""
+    outs = run_ranks(2, "dod", 768, 256, probe=1)
+    for o in outs:
+        assert o["stats"]["h2d_bytes"] == 0
+        bw = o["topology"]["bw_MBps"]
+        assert all(bw[s][d] > 0 for s in range(3) for d in range(3))
+
+
+def test_rank_mode_blas3():
+    run_ranks(4, "blas3", 700, 128)
