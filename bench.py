@@ -18,10 +18,13 @@ Timing: CUDA events on a side stream with a full device synchronize on both side
 K timed steps (the library's work spans its own H2D/D2H/P2P/kernel streams), barrier and
 max over ranks under torchrun.  Inputs (8.6 GB per matrix) are far larger than L2 (126 MB).
 
-Multi-GPU: the library is a single-process multi-GPU runtime (the user's LAPACK matrices
-live in one address space).  Under torchrun rank 0 drives all WORLD_SIZE GPUs
-through xk_init(ngpus=WORLD_SIZE); the other ranks join the barriers and the max-over-ranks
-timing.  Total work is fixed as N grows: "scaling": "strong".
+Multi-GPU: under torchrun the library runs in rank mode -- one process per GPU.  The host
+matrices live in /dev/shm file mappings shared by the processes; every xk call is
+collective; each process executes its own GPU's records of the identical plan (peer tiles
+pulled through CUDA IPC, cross-process order by per-record completion flags).  Each rank
+times its own GPU with CUDA events; the max over ranks is reported.  Total work is fixed
+as the GPU count grows: "scaling": "strong".  (--gpus G without torchrun: one process
+drives G GPUs, the paper's single-process library.)
 
 --impl reference: the CPU oracle (oracle/oracle.c, plain triple loop) timed on the host
 cores on bounded row slabs of the same workload (the reference arm of this tier).
@@ -50,7 +53,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="xk", choices=["xk", "reference"])
-    ap.add_argument("--n", type=int, default=N_DEFAULT)
+    ap.add_argument("--n", "--size", dest="n", type=int, default=N_DEFAULT)
     ap.add_argument("--tile", type=int, default=T_DEFAULT)
     ap.add_argument("--topo", default="ranked")
     ap.add_argument("--optimistic", type=int, default=1)
@@ -77,9 +80,11 @@ def dist_setup(backend=None):
         import torch.distributed as dist
         backend = backend or os.environ.get("XK_DIST_BACKEND", "nccl")
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        if backend == "nccl":
-            lr = int(os.environ.get("LOCAL_RANK", rank))
+        lr = int(os.environ.get("LOCAL_RANK", rank))
+        if torch.cuda.is_available():  # this process's GPU (ranks share it on a one-GPU box)
+            lr = lr % torch.cuda.device_count()
             torch.cuda.set_device(lr)
+        if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
             _HOST_GROUP = dist.new_group(backend="gloo")
         else:
@@ -262,122 +267,159 @@ def run_reference(args, rank, ws):
     print(json.dumps(line), flush=True)
 
 
-def run_xk(args, rank, ws):
+def share_inputs(N, rank, ws):
+    """Host matrices for the run.  One process: plain numpy arrays.  Rank mode (one process
+    per GPU): file mappings in /dev/shm that every process maps (the library's "host
+    memory" is shared by its processes); rank 0 fills them, the others map them after a
+    barrier.  Returns (A, B, C, paths)."""
+    import inputs
+    if ws == 1:
+        A, B, C = make_inputs(N)
+        return A, B, C, []
+    import torch.distributed as dist
+    import paper_conf_sc_gautierl21_b200 as xk
+    obj = [xk.new_session_path("xkbench") if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=_HOST_GROUP)
+    base = obj[0]
+    paths = [base + s for s in (".A", ".B", ".C")]
+    if rank == 0:
+        mats = [xk.shared_matrix(p, N, N, create=True) for p in paths]
+        for M, seed in zip(mats, (inputs.SEED_A, inputs.SEED_B, inputs.SEED_C)):
+            inputs.uniform(seed, N, N, out=M)
+    barrier(ws)
+    if rank != 0:
+        mats = [xk.shared_matrix(p, N, N, create=False) for p in paths]
+    return mats[0], mats[1], mats[2], paths + [base + ".session"]
+
+
+def sum_over_ranks(vals, ws):
+    if ws == 1:
+        return vals
     import torch
+    import torch.distributed as dist
+    t = torch.tensor(vals, dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=_HOST_GROUP)
+    return t.tolist()
+
+
+def run_xk(args, rank, ws):
+    """ws == 1: one process drives the GPU(s) (--gpus G > 1 = the single-process multi-GPU
+    runtime).  Under torchrun (ws > 1): rank mode -- one process per GPU, every xk call
+    collective, each process executing its own GPU's part of the identical plan."""
+    import torch
+    import paper_conf_sc_gautierl21_b200 as xk
     G = ws if ws > 1 else args.gpus
     N, T = args.n, args.tile
     flops = 2.0 * N * N * N
-    xk = None
-    if rank == 0:
-        import paper_conf_sc_gautierl21_b200 as xk
-        A, B, C = make_inputs(N)
-        xk.init(ngpus=G, tile=T, topo=args.topo, optimistic=bool(args.optimistic), kstreams=args.kstreams,
-                probe=True)
-        for X in (A, B, C):
-            xk.register(X)
-        topo = xk.get_topology()
+    A, B, C, paths = share_inputs(N, rank, ws)
+    kw = dict(tile=T, topo=args.topo, optimistic=bool(args.optimistic), kstreams=args.kstreams, probe=True)
+    if ws > 1:
+        xk.init(rank=rank, world=ws, session=paths[-1], **kw)
+    else:
+        xk.init(ngpus=G, **kw)
+    for X in (A, B, C):
+        xk.register(X)
+    topo = xk.get_topology()
     timer = DevTimer()
     clocks = ClockSampler()
 
     # ---------------- value: data-on-device (A, B, C resident in HBM)
-    if rank == 0:
-        for X in (A, B, C):
-            xk.memory_prefetch_async(N, N, X, N)
+    for X in (A, B, C):
+        xk.memory_prefetch_async(N, N, X, N)
+    xk.sync()
+    for _ in range(args.warmup):
+        xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
         xk.sync()
-        for _ in range(args.warmup):
-            xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-            xk.sync()
-        xk.reset_stats()
+    xk.reset_stats()
     barrier(ws)
-    clocks.start()
-    timer.start()
     if rank == 0:
-        for _ in range(args.steps):
-            xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-            xk.sync()
-    barrier(ws)
+        clocks.start()
+    timer.start()
+    for _ in range(args.steps):
+        xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
+        xk.sync()
     ms = max_over_ranks(timer.stop_ms(), ws)
-    clk = clocks.stop(G)
-    st_value = xk.get_stats() if rank == 0 else None
+    barrier(ws)
+    clk = clocks.stop(G) if rank == 0 else None
+    launches = int(sum_over_ranks([xk.get_stats()["kernel_launches"]], ws)[0])
     # roofline pass: the same K steps with every grouped launch timed by CUDA events on its
     # kernel stream (timing serialises launches, so each duration is the kernel's own)
-    st = None
-    if rank == 0:
-        xk.reset_stats()
-        xk.set_kernel_timing(True)
-        for _ in range(args.steps):
-            xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-            xk.sync()
-        st = xk.get_stats()
-        xk.set_kernel_timing(False)
-        xk.memory_coherent_sync(N, N, C, N)
-        xk.memory_invalidate(N, N, C, N)
-        xk.memory_invalidate(N, N, A, N)
-        xk.memory_invalidate(N, N, B, N)
+    xk.reset_stats()
+    xk.set_kernel_timing(True)
+    for _ in range(args.steps):
+        xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
+        xk.sync()
+    st = xk.get_stats()
+    xk.set_kernel_timing(False)
+    k_ms, k_n, k_fl = sum_over_ranks([st["kernel_ms_total"], st["kernel_timed_launches"],
+                                      st["kernel_timed_flops"]], ws)
+    xk.memory_coherent_sync(N, N, C, N)
+    for X in (C, A, B):
+        xk.memory_invalidate(N, N, X, N)
     value = args.steps * flops / (ms * 1e-3) / 1e12
 
     # ---------------- e2e: host-resident, H2D + D2H inside the timed region
     e2e = None
     if not args.no_e2e:
-        if rank == 0:
-            for _ in range(max(1, args.warmup - 1)):
-                xk.dgemm("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-            xk.reset_stats()
+        for _ in range(max(1, args.warmup - 1)):
+            xk.dgemm("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
+        xk.reset_stats()
         barrier(ws)
         timer.start()
-        if rank == 0:
-            for _ in range(args.steps):
-                xk.dgemm("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-        barrier(ws)
+        for _ in range(args.steps):
+            xk.dgemm("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
         ms_e2e = max_over_ranks(timer.stop_ms(), ws)
-        if rank == 0:
-            se = xk.get_stats()
-            h2d = sum(se["h2d_bytes"]) // args.steps
-            d2h = sum(se["d2h_bytes"]) // args.steps
-            tf_e2e = args.steps * flops / (ms_e2e * 1e-3) / 1e12
-            bw_h2d = min(topo["bw_MBps"][G][g] for g in range(G)) * 1e6 * G
-            bw_d2h = min(topo["bw_MBps"][g][G] for g in range(G)) * 1e6 * G
-            t_roof = max(flops / (G * FP64_PEAK_TFLOPS * 1e12), h2d / bw_h2d, d2h / bw_d2h)
-            e2e = {"value": tf_e2e, "unit": "TFLOP/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                   "ms_per_step": ms_e2e / args.steps, "p2p_bytes_per_step": sum(se["p2p_in_bytes"]) // args.steps,
-                   "roofline_frac": t_roof / (ms_e2e * 1e-3 / args.steps),
-                   "roofline": "max(F/(G*P64), B_h2d/BW_h2d, B_d2h/BW_d2h) with P64=%.1f TFLOP/s/GPU and the "
-                               "probed PCIe bandwidths" % FP64_PEAK_TFLOPS}
+        se = xk.get_stats()
+        mine = [sum(se["h2d_bytes"]), sum(se["d2h_bytes"]), sum(se["p2p_in_bytes"])]
+        h2d, d2h, p2p = (int(v) // args.steps for v in sum_over_ranks(mine, ws))
+        tf_e2e = args.steps * flops / (ms_e2e * 1e-3) / 1e12
+        bw_h2d = min(topo["bw_MBps"][G][g] for g in range(G)) * 1e6 * G
+        bw_d2h = min(topo["bw_MBps"][g][G] for g in range(G)) * 1e6 * G
+        t_roof = max(flops / (G * FP64_PEAK_TFLOPS * 1e12), h2d / bw_h2d, d2h / bw_d2h)
+        e2e = {"value": tf_e2e, "unit": "TFLOP/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "ms_per_step": ms_e2e / args.steps, "p2p_bytes_per_step": p2p,
+               "roofline_frac": t_roof / (ms_e2e * 1e-3 / args.steps),
+               "roofline": "max(F/(G*P64), B_h2d/BW_h2d, B_d2h/BW_d2h) with P64=%.1f TFLOP/s/GPU and the "
+                           "probed PCIe bandwidths" % FP64_PEAK_TFLOPS}
 
-    if rank != 0:
-        return
-    launches = st_value["kernel_launches"]
-    timed = max(1, st["kernel_timed_launches"])
-    avg_ms = st["kernel_ms_total"] / timed
-    flops_per_launch = st["kernel_timed_flops"] / timed
+    timed = max(1, int(k_n))
+    avg_ms = k_ms / timed
+    flops_per_launch = k_fl / timed
     achieved = flops_per_launch / (avg_ms * 1e-3) / 1e12 if avg_ms > 0 else None
+    mode = "rank mode: one process per GPU" if ws > 1 else "one process"
     roof = {"bound": "tensor", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
             "frac": (achieved / FP64_PEAK_TFLOPS) if achieved else None, "traffic": traffic_from_profiles(T),
             "kernel": "dgemm_tma_kernel (grouped launch; TMA + mbarrier pipeline; FP64 DMMA.8x8x4 via mma.sync.m8n8k4.f64)",
             "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 x 1965 MHz (no FP64 entry in "
                            "MEASURED_PEAKS.json); DMMA microbenchmark on this pool measured 37.07",
             "per_launch": "one grouped launch = a batch of tile tasks, 2*T^3 flops each (T=%d); %.3g flops "
-                          "per launch on average; %d launches timed with CUDA events on their kernel stream in a "
-                          "second pass of the same K steps (launches serialised while timed), avg %.3f ms; "
-                          "share of the step: %.3f" % (T, flops_per_launch, timed, avg_ms,
-                                                       st["kernel_ms_total"] / (ms * 1.0))}
+                          "per launch on average; %d launches (all GPUs) timed with CUDA events on their kernel "
+                          "stream in a second pass of the same K steps (launches serialised while timed), avg "
+                          "%.3f ms; share of the step: %.3f" % (T, flops_per_launch, timed, avg_ms,
+                                                                k_ms / G / (ms * 1.0))}
     line = {"metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": G, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": "DGEMM N=%d (m=n=k), tile %d, NN, alpha=1.5, beta=-0.75, %d GPU(s), grid %s, "
                                    "heuristics %s%s" % (N, T, G, "x".join(map(str, _grid(G))), args.topo,
                                                         "+optimistic" if args.optimistic else ""),
-                       "N": N, "tile": T, "parallelism": "owner-computes 2D block-cyclic %s" % "x".join(map(str, _grid(G))),
+                       "N": N, "tile": T,
+                       "parallelism": "%s; owner-computes 2D block-cyclic %s" % (mode, "x".join(map(str, _grid(G)))),
                        "value_mode": "data-on-device: A,B,C resident (prefetched), xk_dgemm_async + xk_sync per step",
                        "e2e_mode": "xk_dgemm from pinned host memory, all H2D/D2H in the timed region",
                        "l2": "no flush: each matrix is 8.6 GB >> 126 MB L2",
                        "inputs": "splitmix64 uniform [-1,1), seeds A=1 B=2 C=3"},
             "gpu_launches": launches, "clocks": clk, "roofline": roof, "e2e": e2e,
             "topology_MBps": topo["bw_MBps"], "task_rate_mflops": topo["task_rate_mflops"]}
-    if not args.no_cpu_baseline and ws == 1:
+    if rank == 0 and not args.no_cpu_baseline and ws == 1:
         line["cpu_baseline"] = cpu_baseline(N, A, B, C)
     xk.finalize()
-    print(json.dumps(line), flush=True)
+    barrier(ws)
+    if rank == 0:
+        for p in paths:
+            if os.path.exists(p):
+                os.unlink(p)
+        print(json.dumps(line), flush=True)
 
 
 def _grid(G):

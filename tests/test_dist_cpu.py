@@ -1,7 +1,9 @@
 """The N>1 launch path of bench.py on CPU (gloo, world_size 2, 127.0.0.1): rendezvous from
-the torchrun environment variables, barriers, max-over-ranks timing, and the rule that only
-rank 0 drives the (single-process, multi-GPU) library and prints.  The data path itself has
-no collective: the fan-out of tiles is the library's peer forwarding."""
+the torchrun environment variables, barriers, max-over-ranks timing, sums of the per-rank
+byte counters, the host matrices shared by the rank-mode processes (rank 0 generates them
+into /dev/shm file mappings, every rank sees the same bits), and the rule that only rank 0
+prints.  The data path itself has no collective: the fan-out of tiles is the library's
+peer forwarding."""
 import os
 import socket
 import subprocess
@@ -20,6 +22,17 @@ assert ws == 2 and rank == int(os.environ["RANK"])
 bench.barrier(ws)
 mx = bench.max_over_ranks(10.0 + rank, ws)
 assert mx == 11.0, mx
+assert bench.sum_over_ranks([1.0 + rank, 5.0], ws) == [3.0, 10.0]
+# rank-mode host matrices: one generator run on rank 0, the same bits on every rank
+import numpy as np, inputs
+A, B, C, paths = bench.share_inputs(48, rank, ws)
+assert np.array_equal(np.asarray(B), inputs.uniform(inputs.SEED_B, 48, 48))
+assert A.shape == (48, 48) and np.asfortranarray(A).flags.f_contiguous
+assert paths[-1].endswith(".session") and len(set(paths)) == 4
+bench.barrier(ws)
+if rank == 0:
+    for p in paths[:3]:
+        os.unlink(p)
 # reference arm under torchrun: rank 0 alone prints one JSON line, the other exits quietly
 if rank == 0:
     print(json.dumps({"rank": 0, "max": mx}))
