@@ -34,6 +34,8 @@ def main():
     ap.add_argument("--tile", type=int, default=256)
     ap.add_argument("--probe", type=int, default=0)
     ap.add_argument("--arena", type=int, default=1 << 30)
+    ap.add_argument("--topo", default="ranked")
+    ap.add_argument("--optimistic", type=int, default=1)
     args = ap.parse_args()
     r, N, T = args.rank, args.n, args.tile
     out = {"rank": r, "case": args.case, "ok": True, "checks": []}
@@ -81,7 +83,7 @@ def main():
     C0 = {name: np.array(M, order="F") for name, M in mats.items()} if r == 0 else None
 
     xk.init(rank=r, world=args.world, session=args.session, tile=T, probe=bool(args.probe),
-            arena_bytes=args.arena)
+            arena_bytes=args.arena, topo=args.topo, optimistic=bool(args.optimistic))
     if r != 0:
         reopen()
     for M in mats.values():

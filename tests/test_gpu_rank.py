@@ -26,13 +26,14 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run_ranks(world, case, n=1000, tile=256, probe=0, timeout=600):
+def run_ranks(world, case, n=1000, tile=256, probe=0, timeout=600, topo="ranked", optimistic=1):
     with tempfile.TemporaryDirectory(dir="/dev/shm" if os.path.isdir("/dev/shm") else None) as d:
         session = os.path.join(d, "session")
         procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "rank_worker.py"),
                                    "--rank", str(r), "--world", str(world), "--session", session,
                                    "--dir", d, "--case", case, "--n", str(n), "--tile", str(tile),
-                                   "--probe", str(probe), "--arena", str(1 << 30)],
+                                   "--probe", str(probe), "--arena", str(1 << 30), "--topo", topo,
+                                   "--optimistic", str(optimistic)],
                                   stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True, cwd=ROOT)
                  for r in range(world)]
         outs = []
@@ -51,9 +52,9 @@ def run_ranks(world, case, n=1000, tile=256, probe=0, timeout=600):
     return outs
 
 
-def plan_bytes(topo, calls, tile, world):
+def plan_bytes(links, calls, tile, world, **flags):
     """Per-GPU H2D / P2P-in / D2H bytes of the plan, replayed on the CPU planner."""
-    s = xk.PlanSession(topo["bw_MBps"], topo["task_rate_mflops"], tile=tile)
+    s = xk.PlanSession(links["bw_MBps"], links["task_rate_mflops"], tile=tile, **flags)
     h2d, p2p, d2h = [0] * world, [0] * world, [0] * world
     try:
         for c in calls:
@@ -70,12 +71,12 @@ def plan_bytes(topo, calls, tile, world):
     return h2d, p2p, d2h
 
 
-def assert_bytes_follow_plan(outs, calls, tile):
+def assert_bytes_follow_plan(outs, calls, tile, **flags):
     world = len(outs)
-    topo = outs[0]["topology"]
+    links = outs[0]["topology"]
     for o in outs[1:]:
-        assert o["topology"] == topo, "every rank must build the identical link matrix"
-    h2d, p2p, d2h = plan_bytes(topo, calls, tile, world)
+        assert o["topology"] == links, "every rank must build the identical link matrix"
+    h2d, p2p, d2h = plan_bytes(links, calls, tile, world, **flags)
     for o in outs:
         r, st = o["rank"], o["stats"]
         assert (st["h2d_bytes"], st["p2p_in_bytes"], st["d2h_bytes"]) == (h2d[r], p2p[r], d2h[r]), (r, st)
@@ -89,16 +90,20 @@ def addr(i, n):
     return BASE + i * (8 * n * n + (1 << 20))
 
 
-@pytest.mark.parametrize("world", [2, 4])
-def test_rank_mode_gemm_bitwise_and_bytes(world):
+@pytest.mark.parametrize("world,topo,opt", [(2, "ranked", 1), (4, "ranked", 1), (8, "ranked", 1),
+                                             (8, "ranked", 0), (8, "unranked", 0), (8, "home", 1)])
+def test_rank_mode_gemm_bitwise_and_bytes(world, topo, opt):
+    """Every heuristic mode (paper Table II ablations) at 2/4/8 processes: same bits, bytes
+    per GPU as planned."""
     N, T = 1000, 256
-    outs = run_ranks(world, "gemm", N, T)
+    outs = run_ranks(world, "gemm", N, T, topo=topo, optimistic=opt)
     A, B, C, E = (addr(i, N) for i in range(4))
     calls = [xk.make_call(m=N, n=N, k=N, alpha=-2.0, beta=0.5, A=A, lda=N, B=B, ldb=N, C=C, ldc=N, sync=True),
              xk.make_call(transA="T", m=N, n=N, k=N, alpha=1.0, beta=0.0, A=A, lda=N, B=C, ldb=N, C=E, ldc=N,
                           sync=True)]
-    assert_bytes_follow_plan(outs, calls, T)
-    assert sum(o["stats"]["p2p_in_bytes"] for o in outs) > 0, "tiles must be forwarded between processes"
+    assert_bytes_follow_plan(outs, calls, T, topo=topo, optimistic=bool(opt))
+    p2p = sum(o["stats"]["p2p_in_bytes"] for o in outs)
+    assert (p2p == 0) if topo == "home" else (p2p > 0), "tiles are forwarded between processes unless host-first"
 
 
 def test_rank_mode_composition_no_h2d_of_intermediate():
