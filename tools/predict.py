@@ -27,4 +27,20 @@ for box, (bw, rate) in boxes.items():
             row[name] = {"pred_tflops": round(2.0 * N ** 3 / t / 1e12, 2), "h2d_GB": round(h2d, 2)}
         out["%s_N%d" % (box, N)] = row
         print(box, N, json.dumps(row))
+# the north-star configuration (BASELINE configs[4]): N=65536 on 8x B200, tile sweep, full
+# heuristics vs host-first; fraction of 8 x 37.2 TFLOP/s
+bw, rate = boxes["hgx_b200"]
+N = 65536
+for T in (1024, 2048, 4096):
+    call = xk.make_call(m=N, n=N, k=N, alpha=1.5, beta=-0.75, A=1 << 40, lda=N, B=2 << 40, ldb=N, C=3 << 40, ldc=N, sync=True)
+    row = {}
+    for name, topo, opt in (MODES[0], MODES[3]):
+        recs = xk.plan_dump(call, bw, rate_mflops=rate, topo=topo, optimistic=opt, tile=T, cap=1 << 20)
+        t = max(r[12] for r in recs) * 1e-9
+        h2d = sum(r[13] for r in recs if r[1] == 0) / 1e9
+        tf = 2.0 * N ** 3 / t / 1e12
+        row[name] = {"pred_tflops": round(tf, 1), "frac_of_8x_fp64_peak": round(tf / (8 * 37.22), 3),
+                     "h2d_GB": round(h2d, 1)}
+    out["hgx_b200_N65536_T%d" % T] = row
+    print("hgx_b200 N=65536 T=%d" % T, json.dumps(row))
 print(json.dumps(out))
