@@ -1442,6 +1442,15 @@ int Runtime::finalize() {
     std::lock_guard<std::recursive_mutex> lk(mu);
     if (tracing_) trace_stop();
     const bool peer_failed = rank_mode_ && sess_ && sess_->aborted();
+    if (peer_failed && sess_->flags()) {
+        // a peer died mid-call: release every stream still waiting on one of its flags
+        // (values far ahead of any pending seq pass the cyclic GEQ) so the local work drains
+        // and the arena can be freed; the session is unusable from here on
+        const uint32_t v = (uint32_t)(planner_ ? planner_->next_seq() : 0) + (1u << 30);
+        uint32_t *f = sess_->flags();
+        for (uint32_t i = 0; i < kFlagCap; ++i) __atomic_store_n(f + i, v, __ATOMIC_RELAXED);
+        std::atomic_thread_fence(std::memory_order_seq_cst);
+    }
     int rc = peer_failed ? XK_ERR_CUDA : sync_all();
     if (rank_mode_) {
         // close the mappings of the peers' arenas before anyone frees its own

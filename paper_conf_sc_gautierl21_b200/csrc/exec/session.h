@@ -52,7 +52,7 @@ public:
     int open(const std::string &path, int rank, int world, double timeout_s, std::string &err);
     void close(bool unlink_file);
     // All ranks arrive; returns false on abort or timeout.
-    bool barrier(double timeout_s = 1800.0);
+    bool barrier(double timeout_s = 900.0);
     void abort() { if (h_) h_->aborted.store(1); }
     bool aborted() const { return h_ && h_->aborted.load() != 0; }
     SessionHeader *hdr() { return h_; }

@@ -72,6 +72,10 @@ def main():
         mat("E", N, N, lambda M: M.fill(0.0))
         if args.case == "compose":
             mat("D", N, N, lambda M: M.fill(0.0))
+    elif args.case == "big":
+        mat("A", N, N, lambda M: inputs.integers(1, N, N, out=M))
+        mat("B", N, N, lambda M: inputs.integers(2, N, N, out=M))
+        mat("C", N, N, lambda M: inputs.integers(3, N, N, out=M))
     elif args.case == "blas3":
         k = N // 2 + 3
         mat("A", N, k, lambda M: inputs.integers(1, N, k, out=M))
@@ -80,7 +84,8 @@ def main():
         mat("S", N, N, lambda M: inputs.integers(4, N, N, out=M))
         mat("X", N, N, lambda M: inputs.integers(5, N, N, out=M))
         mat("L", N, N, lambda M: inputs.tri_dd(4, N, lower=True, out=M))
-    C0 = {name: np.array(M, order="F") for name, M in mats.items()} if r == 0 else None
+    keep = ("C",) if args.case == "big" else tuple(mats)
+    C0 = {name: np.array(mats[name], order="F") for name in keep} if r == 0 else None
 
     xk.init(rank=r, world=args.world, session=args.session, tile=T, probe=bool(args.probe),
             arena_bytes=args.arena, topo=args.topo, optimistic=bool(args.optimistic))
@@ -110,6 +115,9 @@ def main():
         assert xk.dgemm_async("N", "N", N, N, N, 1.0, m["A"], N, m["B"], N, -1.0, m["C"], N) == 0
         xk.sync()
         xk.memory_coherent_sync(N, N, m["C"], N)
+    elif args.case == "big":
+        # bench.py's launch configuration (alpha, beta, tile) on exact-integer inputs
+        assert xk.dgemm("N", "N", N, N, N, 1.5, m["A"], N, m["B"], N, -0.75, m["C"], N) == 0
     elif args.case == "blas3":
         k = N // 2 + 3
         assert xk.dsyrk("L", "N", N, k, 2.0, m["A"], N, -1.0, m["C"], N) == 0
@@ -137,6 +145,13 @@ def main():
             ref = c["C"].copy(order="F")
             oracle.dgemm("N", "N", N, N, N, 1.0, c["A"], c["B"], -1.0, ref)
             check("C bitwise", np.array_equal(np.asarray(m["C"]), ref))
+        elif args.case == "big":
+            # Freivalds, exact in FP64 (every partial sum is a multiple of 1/4 below 2^51)
+            rng = np.random.default_rng(5)
+            A_, B_, C_ = np.asarray(m["A"]), np.asarray(m["B"]), np.asarray(m["C"])
+            for _ in range(2):
+                x = rng.integers(-4, 5, N).astype(np.float64)
+                check("freivalds", np.array_equal(C_ @ x, 1.5 * (A_ @ (B_ @ x)) - 0.75 * (c["C"] @ x)))
         elif args.case == "compose":
             refD = np.zeros((N, N), order="F")
             oracle.dgemm("N", "N", N, N, N, 1.0, c["A"], c["B"], 0.0, refD)

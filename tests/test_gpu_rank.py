@@ -26,13 +26,13 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run_ranks(world, case, n=1000, tile=256, probe=0, timeout=600, topo="ranked", optimistic=1):
+def run_ranks(world, case, n=1000, tile=256, probe=0, timeout=600, topo="ranked", optimistic=1, arena=1 << 30):
     with tempfile.TemporaryDirectory(dir="/dev/shm" if os.path.isdir("/dev/shm") else None) as d:
         session = os.path.join(d, "session")
         procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "rank_worker.py"),
                                    "--rank", str(r), "--world", str(world), "--session", session,
                                    "--dir", d, "--case", case, "--n", str(n), "--tile", str(tile),
-                                   "--probe", str(probe), "--arena", str(1 << 30), "--topo", topo,
+                                   "--probe", str(probe), "--arena", str(arena), "--topo", topo,
                                    "--optimistic", str(optimistic)],
                                   stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True, cwd=ROOT)
                  for r in range(world)]
@@ -133,3 +133,15 @@ def test_rank_mode_data_on_device_and_probe():
 
 def test_rank_mode_blas3():
     run_ranks(4, "blas3", 700, 128)
+
+
+def test_rank_mode_bench_configuration_freivalds():
+    """bench.py's multi-GPU launch configuration at full size: rank mode, N=32768, T=4096,
+    alpha=1.5, beta=-0.75, 2 processes -- exact-integer inputs, Freivalds check exact in FP64;
+    bytes per rank as planned."""
+    N, T = 32768, 4096
+    outs = run_ranks(2, "big", N, T, timeout=1200, arena=24 << 30)
+    A, B, C = (addr(i, N) for i in range(3))
+    calls = [xk.make_call(m=N, n=N, k=N, alpha=1.5, beta=-0.75, A=A, lda=N, B=B, ldb=N, C=C, ldc=N, sync=True)]
+    assert_bytes_follow_plan(outs, calls, T)
+    assert "freivalds" in outs[0]["checks"]
