@@ -303,12 +303,26 @@ int Runtime::init_rank_mode(const xk_config_t &cfg) {
     XK_CK(cudaDeviceGetAttribute(&bus, cudaDevAttrPciBusId, d.phys));
     XK_CK(cudaDeviceGetAttribute(&dv, cudaDevAttrPciDeviceId, d.phys));
     me.pci = (dom << 16) | (bus << 8) | dv;
+    // everything that shapes the plan must agree, or the processes would execute different
+    // plans (FNV-1a over the fields; kstreams and the like only change local issue)
+    uint64_t hcfg = 1469598103934665603ull;
+    for (int64_t v : {(int64_t)cfg.tile, (int64_t)cfg.topo, (int64_t)cfg.optimistic, (int64_t)cfg.window,
+                      (int64_t)cfg.grid_p, (int64_t)cfg.grid_q, (int64_t)cfg.probe, cfg.task_rate_mflops}) {
+        hcfg ^= (uint64_t)v;
+        hcfg *= 1099511628211ull;
+    }
+    me.plan_cfg = hcfg;
     auto bar = [&](const char *what) {
         if (sess_->barrier(300.0)) return XK_OK;
         set_error(std::string("rank mode: a peer failed or timed out during ") + what);
         return XK_ERR_CUDA;
     };
     if ((rc = bar("init (device ids)"))) return rc;
+    for (int g = 0; g < G; ++g)
+        if (h->rank[g].plan_cfg != me.plan_cfg) {
+            set_error("config: rank mode needs the same tile/topo/optimistic/window/grid/probe/task rate on every rank");
+            return XK_ERR_CONFIG;
+        }
     int share = 0;
     for (int g = 0; g < G; ++g) {
         devs_[g].pci = h->rank[g].pci;

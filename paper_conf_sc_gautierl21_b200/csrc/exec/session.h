@@ -34,6 +34,7 @@ struct SessionRank {
     int64_t bw_to_host;            // bw[rank][host]
     int64_t bw_local;              // bw[rank][rank]
     int64_t rate_mflops;           // FP64 tile-task rate (rank 0's is used)
+    uint64_t plan_cfg;             // hash of the plan-shaping configuration (must agree)
 };
 
 struct SessionHeader {

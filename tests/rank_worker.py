@@ -87,6 +87,17 @@ def main():
     keep = ("C",) if args.case == "big" else tuple(mats)
     C0 = {name: np.array(mats[name], order="F") for name in keep} if r == 0 else None
 
+    if args.case == "mismatch":
+        # rank 1 asks for another tile size: every rank must refuse (different plans)
+        try:
+            xk.init(rank=r, world=args.world, session=args.session, tile=T * (2 if r == 1 else 1),
+                    probe=False, arena_bytes=args.arena)
+            out["init_error"] = 0
+            xk.finalize()
+        except xk.XKError as e:
+            out["init_error"] = e.code
+        print(json.dumps(out), flush=True)
+        return
     xk.init(rank=r, world=args.world, session=args.session, tile=T, probe=bool(args.probe),
             arena_bytes=args.arena, topo=args.topo, optimistic=bool(args.optimistic))
     if r != 0:

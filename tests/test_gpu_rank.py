@@ -145,3 +145,10 @@ def test_rank_mode_bench_configuration_freivalds():
     calls = [xk.make_call(m=N, n=N, k=N, alpha=1.5, beta=-0.75, A=A, lda=N, B=B, ldb=N, C=C, ldc=N, sync=True)]
     assert_bytes_follow_plan(outs, calls, T)
     assert "freivalds" in outs[0]["checks"]
+
+
+def test_rank_mode_refuses_diverging_configuration():
+    """Ranks whose plan-shaping configuration differs (here the tile size) would execute
+    different plans: xk_init fails with XK_ERR_CONFIG on every rank, nobody hangs."""
+    outs = run_ranks(2, "mismatch", 512, 128, timeout=300)
+    assert [o["init_error"] for o in outs] == [4, 4]
