@@ -5,8 +5,8 @@
 // TRSM/TRMM tile (PLASMA's dtrsm/dtrmm on a tile): recursive blocking on the
 // order of the triangular matrix -- the two half-size triangles recurse, the off-diagonal
 // block is one GEMM on the sm_100a DMMA tile kernel (dgemm_tile.cu), and below 64 a base
-// kernel solves (or multiplies) one vector per thread against the small triangle held in
-// shared memory.  Recursive blocking keeps the substitution backward stable (no explicit
+// kernel solves (or multiplies) one vector per thread, held in registers, against the small
+// triangle held in shared memory (128 vectors per CTA share one triangle load).  Recursive blocking keeps the substitution backward stable (no explicit
 // inverse), so the componentwise residual bound of DESIGN.md reading Q13 holds.
 //
 // Only the triangle op(A) references is read; with diag == 'U' the diagonal is not read.
@@ -30,152 +30,182 @@ __device__ __forceinline__ double opa(const double *A, int64_t lda, bool trans, 
 //   right side: v = a row of B (element stride ldb, vectors 1 apart),   matrix M = op(A)^T
 // LOWER: M is lower triangular (forward substitution / bottom-up product).
 // One launch covers the vectors of every B tile of a batch (all share the triangle).
+#ifndef XK_VPC
+#define XK_VPC 128
+#endif
+constexpr int VPC = XK_VPC;  // vectors (threads) per CTA: the triangle load is shared by all
+static_assert(VPC % 32 == 0 && (NB * NB) % VPC == 0, "VPC: whole warps, triangle split evenly");
 struct BaseBatch {
     int n;                            // tiles
-    int cta_start[kMaxBatch + 1];     // CTAs per tile: ceil(nvec / NB)
+    int cta_start[kMaxBatch + 1];     // CTAs per tile: ceil(nvec / VPC)
     double *B[kMaxBatch];
     int64_t ldb[kMaxBatch], nvec[kMaxBatch];
 };
 
 constexpr int LDM = NB + 2;  // triangle stride in shared memory (16-byte aligned rows)
 
+constexpr int LDV = NB + 2;  // staged vector stride (left side): 16-byte rows, odd in 16-byte units
+constexpr size_t kBaseSmemLeft = (size_t)(NB * LDM + NB + VPC * LDV) * sizeof(double);
+
 template <bool SOLVE, bool LOWER, bool LEFT>
-__global__ void __launch_bounds__(NB) trxm_base_kernel(const __grid_constant__ BaseBatch bb, int n,
-                                                       double alpha, const double *A, int64_t lda,
-                                                       bool mtrans, bool unit) {
-    extern __shared__ double sm[];
+__global__ void __launch_bounds__(VPC) trxm_base_kernel(const __grid_constant__ BaseBatch bb, int n,
+                                                        double alpha, const double *A, int64_t lda,
+                                                        bool mtrans, bool unit) {
     // SOLVE: Ms[c * LDM + i] = M(i, c) (columns contiguous: column-oriented substitution);
     // multiply: Ms[i * LDM + c] = M(i, c) (rows contiguous: row dot products).  Either way
     // the inner loop reads two consecutive entries with one 16-byte shared load, and every
     // thread of the warp reads the same address (broadcast).
-    double *Ms = sm;
-    double(*V)[NB + 1] = reinterpret_cast<double(*)[NB + 1]>(sm + NB * LDM);  // V[element][vector]
-    double *rd = sm + NB * LDM + NB * (NB + 1);                               // 1 / M(l, l)
+    extern __shared__ __align__(16) double smem_base[];
+    double *Ms = smem_base;
+    double *rd = Ms + NB * LDM;  // 1 / M(l, l)
+    double *V = rd + NB;         // left side: the CTA's vectors, V[v * LDV + e]
     int q = 0;
 #pragma unroll 1
     while (q + 1 < bb.n && (int)blockIdx.x >= bb.cta_start[q + 1]) ++q;
     double *B = bb.B[q];
     const int64_t ldb = bb.ldb[q], nvec = bb.nvec[q];
-    const int64_t es = LEFT ? 1 : ldb, vs = LEFT ? ldb : 1;
     const int tid = threadIdx.x;
-    const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * NB;
+    const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * VPC;
+    const int nv = (int)((nvec - v0) < VPC ? (nvec - v0) : VPC);
     // triangle of M into shared memory, padded to NB with the identity (only the referenced
-    // part of A is read).  The kernel is latency-bound, so every load of a phase is issued
-    // before the first shared store (fully unrolled, one element per thread per column:
-    // coalesced along the stored-contiguous direction of A for either transposition).
-    const int nv = (int)((nvec - v0) < NB ? (nvec - v0) : NB);
+    // part of A is read); consecutive threads read along the stored-contiguous direction,
+    // every load in flight before the first shared store (latency-bound phase)
     {
-        double t[NB];
+        double t[NB * NB / VPC];
 #pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            const int i = mtrans ? k : tid, c = mtrans ? tid : k;  // M(i, c); A contiguous in tid
+        for (int k = 0; k < NB * NB / VPC; ++k) {
+            const int e = tid + k * VPC, f = e % NB, s2 = e / NB;
+            const int i = mtrans ? s2 : f, c = mtrans ? f : s2;  // M(i, c); A contiguous in f
             const bool in = LOWER ? (i > c) : (i < c);
-            double x = (i == c) ? 1.0 : 0.0;
-            if (i < n && c < n && (in || (i == c && !unit))) x = opa(A, lda, mtrans, i, c);
-            t[k] = x;
+            double v = (i == c) ? 1.0 : 0.0;
+            if (i < n && c < n && (in || (i == c && !unit))) v = opa(A, lda, mtrans, i, c);
+            t[k] = v;
         }
 #pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            const int i = mtrans ? k : tid, c = mtrans ? tid : k;
+        for (int k = 0; k < NB * NB / VPC; ++k) {
+            const int e = tid + k * VPC, f = e % NB, s2 = e / NB;
+            const int i = mtrans ? s2 : f, c = mtrans ? f : s2;
             Ms[SOLVE ? c * LDM + i : i * LDM + c] = t[k];
             if (SOLVE && i == c) rd[i] = 1.0 / t[k];
         }
-        // vectors of this CTA (coalesced along the contiguous direction of B), zero-padded
-#pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            if (LEFT) {  // element e = tid of vector k
-                t[k] = (tid < n && k < nv) ? B[tid + (v0 + k) * vs] : 0.0;
-            } else {     // vector tid, element k
-                t[k] = (k < n && tid < nv) ? B[(v0 + tid) * vs + k * es] : 0.0;
-            }
-        }
-#pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            if (LEFT) V[tid][k] = t[k];
-            else V[k][tid] = t[k];
-        }
     }
-    __syncthreads();
-    {
-        // one vector per thread, held in registers; every loop is fully unrolled so the
-        // indices are compile-time and independent updates interleave (ILP)
-        const int v = tid;
-        double x[NB];
-#pragma unroll
-        for (int i = 0; i < NB; ++i) x[i] = V[i][v];
-        if (SOLVE) {
-#pragma unroll
-            for (int i = 0; i < NB; ++i) x[i] *= alpha;
-            if (LOWER) {  // column-oriented forward substitution: x_i -= M_il x_l, l ascending
-#pragma unroll
-                for (int l = 0; l < NB; ++l) {
-                    if (!unit) x[l] *= rd[l];
-                    const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
-#pragma unroll
-                    for (int p = (l + 1) / 2; p < NB / 2; ++p) {
-                        const double2 m2 = col[p];
-                        if (2 * p > l) x[2 * p] -= m2.x * x[l];
-                        x[2 * p + 1] -= m2.y * x[l];
-                    }
-                }
-            } else {      // back substitution, l descending
-#pragma unroll
-                for (int l = NB - 1; l >= 0; --l) {
-                    if (!unit) x[l] *= rd[l];
-                    const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
-#pragma unroll
-                    for (int p = 0; 2 * p < l; ++p) {
-                        const double2 m2 = col[p];
-                        x[2 * p] -= m2.x * x[l];
-                        if (2 * p + 1 < l) x[2 * p + 1] -= m2.y * x[l];
-                    }
-                }
-            }
-        } else {
-            if (LOWER) {  // bottom-up: row i only reads x_0..x_i, still unmodified
-#pragma unroll
-                for (int i = NB - 1; i >= 0; --i) {
-                    const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
-                    double s = 0.0;
-#pragma unroll
-                    for (int p = 0; 2 * p <= i; ++p) {
-                        const double2 m2 = row[p];
-                        s += m2.x * x[2 * p];
-                        if (2 * p + 1 <= i) s += m2.y * x[2 * p + 1];
-                    }
-                    x[i] = alpha * s;
-                }
-            } else {      // top-down: row i only reads x_i..x_NB-1, still unmodified
-#pragma unroll
-                for (int i = 0; i < NB; ++i) {
-                    const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
-                    double s = 0.0;
-#pragma unroll
-                    for (int p = i / 2; p < NB / 2; ++p) {
-                        const double2 m2 = row[p];
-                        if (2 * p >= i) s += m2.x * x[2 * p];
-                        s += m2.y * x[2 * p + 1];
-                    }
-                    x[i] = alpha * s;
-                }
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < NB; ++i) V[i][v] = x[i];
-    }
-    __syncthreads();
+    double x[NB];
     if (LEFT) {
-#pragma unroll 16
-        for (int r = tid; r < n * nv; r += NB) {
-            int e = r % n, v = r / n;
-            B[e + (v0 + v) * vs] = V[e][v];
+        // vectors are columns of B (contiguous): a warp loads whole columns, 16 bytes per
+        // lane (fully coalesced), into the staging area; each thread then takes its own
+        const int w = tid >> 5, lane = tid & 31;
+        double2 u[32];  // VPC / 32 warps x 32 columns each = VPC vectors
+#pragma unroll
+        for (int k = 0; k < 32; ++k) {
+            const int v = w * 32 + k, e = 2 * lane;
+            double2 z = make_double2(0.0, 0.0);
+            if (v < nv && e < n) {
+                const double *src = B + (v0 + v) * ldb + e;
+                if (e + 1 < n) z = *reinterpret_cast<const double2 *>(src);
+                else z.x = src[0];
+            }
+            u[k] = z;
+        }
+#pragma unroll
+        for (int k = 0; k < 32; ++k) {
+            const int v = w * 32 + k;
+            *reinterpret_cast<double2 *>(V + v * LDV + 2 * lane) = u[k];
+        }
+        __syncthreads();
+#pragma unroll
+        for (int p = 0; p < NB / 2; ++p) {
+            const double2 z = *reinterpret_cast<const double2 *>(V + tid * LDV + 2 * p);
+            x[2 * p] = z.x;
+            x[2 * p + 1] = z.y;
         }
     } else {
-#pragma unroll 16
-        for (int r = tid; r < n * nv; r += NB) {
-            int v = r % nv, e = r / nv;
-            B[(v0 + v) * vs + e * es] = V[e][v];
+        // vectors are rows of B: consecutive threads read consecutive addresses
+        const bool active = tid < nv;
+        const double *p = B + (v0 + tid);
+#pragma unroll
+        for (int i = 0; i < NB; ++i, p += ldb) x[i] = (active && i < n) ? *p : 0.0;
+    }
+    __syncthreads();
+    if (SOLVE) {
+#pragma unroll
+        for (int i = 0; i < NB; ++i) x[i] *= alpha;
+        if (LOWER) {  // column-oriented forward substitution: x_i -= M_il x_l, l ascending
+#pragma unroll
+            for (int l = 0; l < NB; ++l) {
+                if (!unit) x[l] *= rd[l];
+                const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
+#pragma unroll
+                for (int p = (l + 1) / 2; p < NB / 2; ++p) {
+                    const double2 m2 = col[p];
+                    if (2 * p > l) x[2 * p] -= m2.x * x[l];
+                    x[2 * p + 1] -= m2.y * x[l];
+                }
+            }
+        } else {      // back substitution, l descending
+#pragma unroll
+            for (int l = NB - 1; l >= 0; --l) {
+                if (!unit) x[l] *= rd[l];
+                const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
+#pragma unroll
+                for (int p = 0; 2 * p < l; ++p) {
+                    const double2 m2 = col[p];
+                    x[2 * p] -= m2.x * x[l];
+                    if (2 * p + 1 < l) x[2 * p + 1] -= m2.y * x[l];
+                }
+            }
         }
+    } else {
+        if (LOWER) {  // bottom-up: row i only reads x_0..x_i, still unmodified
+#pragma unroll
+            for (int i = NB - 1; i >= 0; --i) {
+                const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
+                double s = 0.0;
+#pragma unroll
+                for (int p = 0; 2 * p <= i; ++p) {
+                    const double2 m2 = row[p];
+                    s += m2.x * x[2 * p];
+                    if (2 * p + 1 <= i) s += m2.y * x[2 * p + 1];
+                }
+                x[i] = alpha * s;
+            }
+        } else {      // top-down: row i only reads x_i..x_NB-1, still unmodified
+#pragma unroll
+            for (int i = 0; i < NB; ++i) {
+                const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
+                double s = 0.0;
+#pragma unroll
+                for (int p = i / 2; p < NB / 2; ++p) {
+                    const double2 m2 = row[p];
+                    if (2 * p >= i) s += m2.x * x[2 * p];
+                    s += m2.y * x[2 * p + 1];
+                }
+                x[i] = alpha * s;
+            }
+        }
+    }
+    if (LEFT) {
+        // back through the staging area so that every warp stores whole columns
+#pragma unroll
+        for (int p = 0; p < NB / 2; ++p)
+            *reinterpret_cast<double2 *>(V + tid * LDV + 2 * p) = make_double2(x[2 * p], x[2 * p + 1]);
+        __syncthreads();
+        const int w = tid >> 5, lane = tid & 31;
+#pragma unroll
+        for (int k = 0; k < 32; ++k) {
+            const int v = w * 32 + k, e = 2 * lane;
+            if (v < nv && e < n) {
+                const double2 z = *reinterpret_cast<const double2 *>(V + v * LDV + e);
+                double *dst = B + (v0 + v) * ldb + e;
+                if (e + 1 < n) *reinterpret_cast<double2 *>(dst) = z;
+                else dst[0] = z.x;
+            }
+        }
+    } else if (tid < nv) {
+        double *p = B + (v0 + tid);
+        asm volatile("mov.b64 %0, %0;" : "+l"(p));  // opaque: no CSE with the load addresses
+#pragma unroll
+        for (int i = 0; i < NB; ++i, p += ldb)
+            if (i < n) *p = x[i];
     }
 }
 
@@ -201,17 +231,17 @@ inline const double *opa_block(const double *A, int64_t lda, bool trans, int64_t
 template <bool SOLVE, bool LOWER, bool LEFT>
 cudaError_t base_launch(const BaseBatch &bb, unsigned grid, int n, double alpha, const double *A,
                         int64_t lda, bool mtrans, bool unit, cudaStream_t st) {
-    constexpr size_t smem = (NB * LDM + NB * (NB + 1) + NB) * sizeof(double);
     auto kern = trxm_base_kernel<SOLVE, LOWER, LEFT>;
+    const size_t smem = LEFT ? kBaseSmemLeft : (size_t)(NB * LDM + NB) * sizeof(double);
     static unsigned attr_set = 0;  // per instantiation, one bit per device
     int dev = 0;
     cudaGetDevice(&dev);
     if (!(attr_set & (1u << dev))) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBaseSmemLeft);
         if (e != cudaSuccess) return e;
         attr_set |= 1u << dev;
     }
-    kern<<<grid, NB, smem, st>>>(bb, n, alpha, A, lda, mtrans, unit);
+    kern<<<grid, VPC, smem, st>>>(bb, n, alpha, A, lda, mtrans, unit);
     return cudaGetLastError();
 }
 
@@ -225,7 +255,7 @@ cudaError_t base(const TriOp &o, int64_t n, const Tiles &T, double alpha, const 
         bb.B[q] = T.B[q];
         bb.ldb[q] = T.ldb[q];
         bb.nvec[q] = T.other[q];
-        total += (int)((T.other[q] + NB - 1) / NB);
+        total += (int)((T.other[q] + VPC - 1) / VPC);
     }
     bb.cta_start[T.n] = total;
     if (total == 0) return cudaSuccess;
