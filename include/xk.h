@@ -301,6 +301,17 @@ void xk_plan_session_destroy(xk_plan_session_t *s);
 int xk_plan_dump(const xk_call_t *call, const xk_topo_t *topo, const xk_flags_t *flags,
                  xk_plan_rec_t *out, int64_t cap, int64_t *n_out);
 
+/* ------------------------------------------------------------------ rank-mode session */
+/* The host side of rank mode's synchronisation, without CUDA (for CPU tests and tools):
+ * joins the session file `path` as `rank` of `world` (rank 0 creates it and removes it at
+ * the end), passes `rounds` barriers, and writes into flags_out[r] (r < rounds) the number of
+ * ranks that had arrived at round r when this rank left it (every rank must see `world`).
+ * With abort_at >= 0 this rank marks the session aborted instead of arriving at round
+ * abort_at; the others then fail.  Returns 0, XK_ERR_CONFIG (cannot create/join), or
+ * XK_ERR_CUDA (a barrier failed: peer aborted or timeout_s elapsed). */
+int xk_session_selftest(const char *path, int rank, int world, int rounds, int abort_at,
+                        double timeout_s, int *flags_out);
+
 /* ------------------------------------------------------------------ kernel-level entry */
 /* One tile task on device memory, for kernel parity tests and the roofline bench:
  * D = alpha*op(A)*op(B) + beta*C on compact column-major tiles (ld = rows),

@@ -106,6 +106,13 @@ def new_session_path(tag="xk"):
     return os.path.join(d, "%s_%d_%s" % (tag, os.getpid(), os.urandom(6).hex()))
 
 
+def session_selftest(path, rank, world, rounds, abort_at=-1, timeout_s=60.0):
+    """Host side of rank mode's synchronisation (no CUDA): returns (rc, arrivals per round)."""
+    out = (ctypes.c_int * max(1, rounds))()
+    rc = lib().xk_session_selftest(os.fsencode(path), rank, world, rounds, abort_at, timeout_s, out)
+    return rc, list(out)[:rounds]
+
+
 def shared_matrix(path, rows, cols, create):
     """A column-major float64 host matrix backed by a file mapping (MAP_SHARED) that every
     rank-mode process maps: the "host memory" of the library's processes.  Plumbing only --

@@ -124,6 +124,8 @@ _SIGS = [
     ("xk_plan_session_call", c_int, [vp, ctypes.POINTER(Call), ctypes.POINTER(PlanRec), i64,
                                      ctypes.POINTER(i64)]),
     ("xk_plan_session_destroy", None, [vp]),
+    ("xk_session_selftest", c_int, [ctypes.c_char_p, c_int, c_int, c_int, c_int, c_double,
+                                    ctypes.POINTER(c_int)]),
     ("xk_plan_dump", c_int, [ctypes.POINTER(Call), ctypes.POINTER(Topo), ctypes.POINTER(Flags),
                              ctypes.POINTER(PlanRec), i64, ctypes.POINTER(i64)]),
     ("xk_dgemm_tile_device", c_int, [c_char, c_char, i64, i64, i64, _D, vp, i64, vp, i64, _D, vp,

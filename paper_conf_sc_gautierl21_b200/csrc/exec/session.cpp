@@ -168,3 +168,32 @@ void Session::close(bool unlink_file) {
 }
 
 }  // namespace xk
+
+// Round r: every rank adds 1 to a per-round counter in the flag area (host memory only),
+// then waits at the barrier; after it, all `world` increments must be visible.
+extern "C" int xk_session_selftest(const char *path, int rank, int world, int rounds, int abort_at,
+                                   double timeout_s, int *flags_out) {
+    if (!path || world < 1 || world > XK_MAX_GPUS || rank < 0 || rank >= world || rounds < 0) return XK_ERR_CONFIG;
+    xk::Session s;
+    std::string err;
+    int rc = s.open(path, rank, world, timeout_s, err);
+    if (rc) return rc;
+    uint32_t *cnt = s.flags();
+    for (int r = 0; r < rounds; ++r) {
+        if (r == abort_at) {
+            s.abort();
+            s.close(false);
+            return XK_OK;
+        }
+        __atomic_fetch_add(cnt + r, 1u, __ATOMIC_ACQ_REL);
+        if (!s.barrier(timeout_s)) {
+            s.close(rank == 0);
+            return XK_ERR_CUDA;
+        }
+        if (flags_out) flags_out[r] = (int)__atomic_load_n(cnt + r, __ATOMIC_ACQUIRE);
+    }
+    // nobody unmaps before the last reader is done, then rank 0 removes the file
+    const bool ok = s.barrier(timeout_s);
+    s.close(rank == 0);
+    return ok ? XK_OK : XK_ERR_CUDA;
+}
