@@ -839,6 +839,18 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
     const bool fwd = solve ? (left == elow) : (left != elow);
     const int64_t nsteps = tk;
     const int64_t other = left ? tn : tm;  // tiles along the untouched dimension
+    // update window (reading R10) only when B has to come from the host: with every tile
+    // of B already current on a GPU (data-on-device, composition) PCIe does not bind and the
+    // plain right-looking order (window = every step) keeps more updates in flight
+    bool b_on_gpus = true;
+    for (int64_t j = 0; j < tn && b_on_gpus; ++j)
+        for (int64_t i = 0; i < tm && b_on_gpus; ++i) {
+            const Entry &e = entries_[key_of(mc, i, j)];
+            bool cur = false;
+            for (const NodeCopy &g : e.gpu) cur = cur || (g.present && g.ver == e.ver);
+            b_on_gpus = cur;
+        }
+    const int64_t Dw = b_on_gpus ? nsteps : 2 * (left ? flags_.P : flags_.Q);
     for (int64_t s = 0; s < nsteps; ++s) {
         const int64_t kx = fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
         const double a_s = solve ? ((s == 0) ? c.alpha : 1.0) : c.alpha;
@@ -935,9 +947,15 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
                 g.m = mt; g.n = nt; g.k = kt;
                 g.flops = 2 * mt * nt * kt;
                 // lookahead (reading R9): the row (col) the next step solves is updated first,
-                // so its diagonal solve can run while the other updates of this step proceed
-                const int64_t ph = (r == (fwd ? kx + 1 : kx - 1)) ? 1 : 2;
-                int64_t sk[5] = {s, ph, (bi + bj + s) % tmod, bi, bj};
+                // so its diagonal solve can run while the other updates of this step proceed.
+                // Update window (reading R10): the row solved at step sr is updated by step s
+                // at time u = max(s, sr - D), D = 2 x the grid extent along the solved
+                // dimension; within a time, rows nearest the front first, then s ascending
+                // (every tile's chain keeps its order: results are those of right-looking)
+                const int64_t sr = fwd ? r : nsteps - 1 - r;
+                const int64_t u = std::max<int64_t>(s, sr - Dw);
+                const int64_t ph = (sr == s + 1) ? 1 : 2;
+                int64_t sk[5] = {u, ph, sr * nsteps + s, (bi + bj + s) % tmod, o};
                 std::copy(sk, sk + 5, g.skey);
                 tasks.push_back(g);
             }

@@ -396,6 +396,10 @@ class Model:
             return self.tile(A, lda, q, r) if tr else self.tile(A, lda, r, q)
         fwd = (left == elow) if solve else (left != elow)
         other = tn if left else tm
+        # R10 window only when B must come from the host (some tile not current on a GPU)
+        b_on_gpus = all(any(c.ver == tl.ver for c in tl.gpus.values())
+                        for tl in (self.tile(C, ldc, i, j) for j in range(tn) for i in range(tm)))
+        D = tk if b_on_gpus else 2 * (self.P if left else self.Q)
         for s in range(tk):
             kx = s if fwd else tk - 1 - s
             for o in range(other):
@@ -433,9 +437,13 @@ class Model:
                         ins = [(opA(r, kx), 0), (self.tile(C, ldc, kx, bj), 2), (ot, 2)]
                     else:
                         ins = [(self.tile(C, ldc, bi, kx), 2), (opA(kx, r), 0), (ot, 2)]
-                    # lookahead (R9): the next step's row (column) is updated first
-                    ph = 1 if r == (kx + 1 if fwd else kx - 1) else 2
-                    tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins, (s, ph, (bi + bj + s) % tmod, bi, bj),
+                    # lookahead (R9): the next step's row (column) is updated first;
+                    # update window (R10): row solved at step sr is updated by step s at time
+                    # u = max(s, sr - D), D = 2 x grid extent along the solved dimension
+                    sr = r if fwd else tk - 1 - r
+                    u = max(s, sr - D)
+                    ph = 1 if sr == s + 1 else 2
+                    tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins, (u, ph, sr * tk + s, (bi + bj + s) % tmod, o),
                                             2 * mt * nt * kt, s))
         return tasks
 

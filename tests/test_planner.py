@@ -400,28 +400,34 @@ def test_beta_deferral_structure():
 
 @pytest.mark.parametrize("uplo", ["L", "U"])
 def test_trsm_lookahead_order(uplo):
-    """Reading R9 (lookahead): in each step of the tiled TRSM the updates of the row the next
-    step solves come first, right after the step's diagonal solves, so the next diagonal
-    solve depends only on the first updates of the step."""
-    T, t = 4, 5
+    """Readings R9 + R10 on one GPU (D = 2): at time u come the diagonal solves of step u,
+    then the update of the row step u+1 solves by step u (lookahead), then the catch-up
+    updates of the row solved at step u+D by every step s <= u (s ascending) -- far rows are
+    updated just before they are needed, not all in step 0; every tile's chain keeps s
+    ascending.  The expected sequence is written out from the rule, independently of the
+    planner's sort keys."""
+    T, t, D = 4, 5, 2
     N = T * t
     recs = xk.plan_dump(xk.make_call(routine=pm.DTRSM, side="L", uplo=uplo, transA="N", diag="N", m=N, n=N,
                                      alpha=1.0, A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True), uniform(1), tile=T)
     tasks = [r for r in recs if r[1] == pm.TASK]
-    order = list(range(t)) if uplo == "L" else list(range(t - 1, -1, -1))
-    pos = 0
-    for s, kx in enumerate(order):
-        diag = tasks[pos:pos + t]
-        assert all(r[15] == pm.OP_TRSM_DIAG and r[3] == kx for r in diag)
-        pos += t
-        nupd = t * (t - 1 - s)
-        upd = tasks[pos:pos + nupd]
-        assert all(r[15] == pm.OP_GEMM for r in upd)
-        if s + 1 < t:
-            assert all(r[3] == order[s + 1] for r in upd[:t])
-            assert all(r[3] != order[s + 1] for r in upd[t:])
-        pos += nupd
-    assert pos == len(tasks)
+    order = list(range(t)) if uplo == "L" else list(range(t - 1, -1, -1))  # row solved at step s
+    expect = []
+    for u in range(t):
+        expect.append(("diag", order[u], u))
+        if u + 1 < t:
+            expect.append(("upd", order[u + 1], u))
+        sr = u + D  # with D = 2 the only catch-up row at time u
+        if sr < t:
+            expect += [("upd", order[sr], s) for s in range(u + 1)]
+    got = []
+    for r in tasks:
+        kind = "diag" if r[15] == pm.OP_TRSM_DIAG else "upd"
+        key = (kind, r[3], r[5])
+        if not got or got[-1] != key:
+            got.append(key)
+    assert got == expect
+    assert len(tasks) == t * t + t * t * (t - 1) // 2
 
 
 def test_trmm_contributions_nearest_first():
@@ -488,3 +494,35 @@ def test_coherent_writebacks_in_completion_order():
         assert len(wb) == (N // T) ** 2 and all(r[1] == pm.D2H for r in wb)
         done = [by_seq[r[14][0]][12] for r in wb]
         assert done == sorted(done) and len(set(done)) > 1
+
+
+@pytest.mark.parametrize("G", [1, 4, 8])
+def test_trsm_window_depends_on_residency(G):
+    """Reading R10 applies only when B must come from the host: with every B tile current on
+    a GPU (prefetched = data-on-device, or produced by an earlier async call) the plan is the
+    right-looking order; a partly resident B keeps the window.  Bit-exact vs the model in all
+    three cases, for both triangles and sides."""
+    bw = TOPOS["uniform"](G)
+    flags = dict(topo="ranked", optimistic=True, window=2, tile=4)
+    N = 24
+    for side, uplo in itertools.product("LR", "LU"):
+        trsm = dict(routine=pm.DTRSM, side=side, uplo=uplo, transA="N", diag="N", m=N, n=N, alpha=1.5,
+                    A=A_ADDR, lda=N, C=B_ADDR, ldc=N, sync=False)
+        for pre in (None, (N, N), (N // 2, N)):
+            calls = []
+            if pre:
+                calls.append(dict(routine=pm.PREFETCH, m=pre[0], n=pre[1], C=B_ADDR, ldc=N))
+            calls += [trsm, dict(routine=pm.COHERENT, m=N, n=N, C=B_ADDR, ldc=N), dict(routine=pm.SYNC)]
+            got, exp = both(bw, flags, calls)
+            assert got == exp, (G, side, uplo, pre)
+    # on one GPU the resident case is plain right-looking: every update of step s comes
+    # before the diagonal solve of step s+1 ... and the host-resident case is not
+    if G == 1:
+        def update_steps(recs):
+            return [r[5] for r in recs if r[1] == pm.TASK]
+        trsm = dict(routine=pm.DTRSM, side="L", uplo="L", transA="N", diag="N", m=N, n=N, alpha=1.5,
+                    A=A_ADDR, lda=N, C=B_ADDR, ldc=N, sync=False)
+        res, _ = both(bw, flags, [dict(routine=pm.PREFETCH, m=N, n=N, C=B_ADDR, ldc=N), trsm])
+        host, _ = both(bw, flags, [trsm])
+        assert update_steps(res[1]) == sorted(update_steps(res[1]))
+        assert update_steps(host[0]) != sorted(update_steps(host[0]))
