@@ -269,27 +269,48 @@ def run_reference(args, rank, ws):
 
 def share_inputs(N, rank, ws):
     """Host matrices for the run.  One process: plain numpy arrays.  Rank mode (one process
-    per GPU): file mappings in /dev/shm that every process maps (the library's "host
-    memory" is shared by its processes); rank 0 fills them, the others map them after a
-    barrier.  Returns (A, B, C, paths)."""
+    per GPU): file mappings every process maps (the library's "host memory" is shared by its
+    processes) -- files in /dev/shm when it has room, else anonymous memfds that the other
+    ranks open through /proc/<rank 0>/fd (a small /dev/shm mount must not cap the run);
+    rank 0 fills them, the others map them after a barrier.  Returns (A, B, C, paths) with
+    the session-file path last; only real files in the list are unlinked at the end."""
     import inputs
     if ws == 1:
         A, B, C = make_inputs(N)
         return A, B, C, []
     import torch.distributed as dist
     import paper_conf_sc_gautierl21_b200 as xk
-    obj = [xk.new_session_path("xkbench") if rank == 0 else None]
-    dist.broadcast_object_list(obj, src=0, group=_HOST_GROUP)
-    base = obj[0]
-    paths = [base + s for s in (".A", ".B", ".C")]
+    obj = [None]
     if rank == 0:
-        mats = [xk.shared_matrix(p, N, N, create=True) for p in paths]
+        base = xk.new_session_path("xkbench")
+        need = 3 * N * N * 8
+        try:
+            st = os.statvfs("/dev/shm")
+            room = st.f_bavail * st.f_frsize > 1.1 * need
+        except OSError:
+            room = False
+        if room and os.environ.get("XK_SHARE") != "memfd":
+            paths = [base + s for s in (".A", ".B", ".C")]
+            for p in paths:
+                xk.shared_matrix(p, N, N, create=True)
+        else:
+            global _MEMFDS
+            _MEMFDS = [os.memfd_create("xkbench" + s) for s in "ABC"]
+            for fd in _MEMFDS:
+                os.ftruncate(fd, N * N * 8)
+            paths = ["/proc/%d/fd/%d" % (os.getpid(), fd) for fd in _MEMFDS]
+        obj = [paths + [base + ".session"]]
+    dist.broadcast_object_list(obj, src=0, group=_HOST_GROUP)
+    paths = obj[0]
+    mats = [xk.shared_matrix(p, N, N, create=False) for p in paths[:3]]
+    if rank == 0:
         for M, seed in zip(mats, (inputs.SEED_A, inputs.SEED_B, inputs.SEED_C)):
             inputs.uniform(seed, N, N, out=M)
     barrier(ws)
-    if rank != 0:
-        mats = [xk.shared_matrix(p, N, N, create=False) for p in paths]
-    return mats[0], mats[1], mats[2], paths + [base + ".session"]
+    return mats[0], mats[1], mats[2], [p for p in paths if not p.startswith("/proc/")]
+
+
+_MEMFDS = []
 
 
 def sum_over_ranks(vals, ws):
