@@ -617,7 +617,7 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
             int64_t mt = std::min(T, n - i * T), nt = std::min(T, n - j * T);
             if (scale_only) {
                 Task t;
-                t.gpu = owner(i, j);
+                t.gpu = owner_tri(i, j, lower, tn);
                 t.op = XK_OP_SCALE;
                 t.tri = dg ? tri : 0;
                 t.out_key = keyC;
@@ -645,7 +645,7 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
                     int xa = (two && s == 1) ? mb : ma, xb = (two && s == 0) ? mb : ma;
                     int keyA = opnd(xa, i, l), keyB = opnd(xb, j, l);
                     Task t;
-                    t.gpu = owner(i, j);
+                    t.gpu = owner_tri(i, j, lower, tn);
                     t.op = dg ? XK_OP_GEMM_TRI : XK_OP_GEMM;
                     t.tri = dg ? tri : 0;
                     t.out_key = keyC;

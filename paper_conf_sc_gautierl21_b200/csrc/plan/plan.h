@@ -99,6 +99,12 @@ public:
     int owner(int64_t i, int64_t j) const {
         return (int)((i % flags_.P) * flags_.Q + (j % flags_.Q));
     }
+    // Owner of tile (i, j) of a triangular output (SYRK/SYR2K, reading R11): the stored
+    // triangle's tiles in column-major order dealt round-robin over the G GPUs
+    int owner_tri(int64_t i, int64_t j, bool lower, int64_t t) const {
+        const int64_t idx = lower ? j * t - j * (j - 1) / 2 + (i - j) : j * (j + 1) / 2 + i;
+        return (int)(idx % topo_.G);
+    }
     const Flags &flags() const { return flags_; }
     int64_t next_seq() const { return seq_; }  // seq of the next record to be emitted
     int link_class(int s, int d) const { return cls_[(size_t)s * (topo_.G + 1) + d]; }

@@ -214,9 +214,15 @@ class Model:
         return out
 
     # ---- task generators: program order, symbolic versions (readings in DESIGN.md)
-    def _task(self, vers, op, i, j, out, ins, skey, flops, tk):
+    def owner_tri(self, i, j, lower, t):
+        """Triangular outputs (SYRK/SYR2K, R11): the stored triangle's tiles in
+        column-major order, dealt round-robin over the GPUs."""
+        idx = j * t - j * (j - 1) // 2 + (i - j) if lower else j * (j + 1) // 2 + i
+        return idx % self.G
+
+    def _task(self, vers, op, i, j, out, ins, skey, flops, tk, gpu=None):
         """ins = [(tile, operand)] in input order; versions read now, output bumped."""
-        t = dict(gpu=self.owner(i, j), op=op, out=out, tk=tk, i=i, j=j, flops=flops, skey=skey,
+        t = dict(gpu=self.owner(i, j) if gpu is None else gpu, op=op, out=out, tk=tk, i=i, j=j, flops=flops, skey=skey,
                  ins=[(tl, vers.get(id(tl), tl.ver), opnd) for (tl, opnd) in ins])
         vers[id(out)] = vers.get(id(out), out.ver) + 1
         t["ver"] = vers[id(out)]
@@ -309,7 +315,8 @@ class Model:
                 mt, nt = min(T, n - i * T), min(T, n - j * T)
                 if scale:
                     ins = [(ct, 2)] if (beta != 0 or dg) else []
-                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
+                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, ins, (0, (i + j) % tmod, i, j, 0), mt * nt, -1,
+                                            gpu=self.owner_tri(i, j, lower, tn)))
                     continue
                 first = True
                 defer = shadow is not None and not dg and self.host_only(ct)  # diagonal: R5
@@ -326,7 +333,8 @@ class Model:
                             ins.append((self.tile(shadow, ldc, i, j), 2))
                         fl = kt * nt * (nt + 1) if dg else 2 * mt * nt * kt
                         tasks.append(self._task(vers, OP_GEMM_TRI if dg else OP_GEMM, i, j, ct, ins,
-                                                (2 * (l + (i + j) % tk) + s, (i + j + l) % tmod, i, j, 0), fl, l))
+                                                (2 * (l + (i + j) % tk) + s, (i + j + l) % tmod, i, j, 0), fl, l,
+                                                gpu=self.owner_tri(i, j, lower, tn)))
                         first = False
                         pos += 1
         return tasks

@@ -43,4 +43,27 @@ for T in (1024, 2048, 4096):
                      "h2d_GB": round(h2d, 1)}
     out["hgx_b200_N65536_T%d" % T] = row
     print("hgx_b200 N=65536 T=%d" % T, json.dumps(row))
+# BASELINE configs[2]/[3] on 8x B200 (N=32768, T=2048): DSYRK / DSYR2K (lower, N) and
+# DTRSM / DTRMM (left, lower, N, non-unit), host-resident, full heuristics vs host-first;
+# per-GPU task-time balance of the owner map (max / mean busy time)
+N, T = 32768, 2048
+fl = {"dsyrk": N * N * (N + 1), "dsyr2k": 2 * N * N * N + N, "dtrsm": N * N * N, "dtrmm": N * N * N}
+rt = {"dsyrk": xk._abi.ROUTINE_DSYRK, "dsyr2k": xk._abi.ROUTINE_DSYR2K, "dtrsm": xk._abi.ROUTINE_DTRSM, "dtrmm": xk._abi.ROUTINE_DTRMM}
+for name in ("dsyrk", "dsyr2k", "dtrsm", "dtrmm"):
+    row = {}
+    for mode, topo, opt in (MODES[0], MODES[3]):
+        call = xk.make_call(routine=rt[name], uplo="L", transA="N", side="L", diag="N", m=N, n=N, k=N,
+                            alpha=1.5, beta=-0.75, A=1 << 40, lda=N, B=2 << 40, ldb=N, C=3 << 40, ldc=N, sync=True)
+        recs = xk.plan_dump(call, bw, rate_mflops=rate, topo=topo, optimistic=opt, tile=T, cap=1 << 20)
+        t = max(r[12] for r in recs) * 1e-9
+        busy = [0] * 8
+        for r in recs:
+            if r[1] == 2:
+                busy[r[7]] += r[12] - r[11]
+        tf = fl[name] / t / 1e12
+        row[mode] = {"pred_tflops": round(tf, 1), "frac_of_8x_fp64_peak": round(tf / (8 * 37.22), 3),
+                     "busy_max_over_mean": round(max(busy) / (sum(busy) / 8), 3),
+                     "h2d_GB": round(sum(r[13] for r in recs if r[1] == 0) / 1e9, 1)}
+    out["hgx_b200_%s_N32768_T2048" % name] = row
+    print("hgx_b200", name, json.dumps(row))
 print(json.dumps(out))
