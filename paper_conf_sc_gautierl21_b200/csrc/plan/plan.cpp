@@ -815,7 +815,7 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             for (int64_t i = 0; i < tm; ++i) {
                 int keyC = key_of(mc, i, j);
                 Task t;
-                t.gpu = owner(i, j);
+                t.gpu = owner_trxm(i, j, left, solve);
                 t.op = XK_OP_SCALE;
                 t.out_key = keyC;
                 t.out_ver = V.bump(keyC);
@@ -860,7 +860,7 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
             // diagonal task on B(kx, o) (left) / B(o, kx) (right)
             Task t;
-            t.gpu = owner(bi, bj);
+            t.gpu = owner_trxm(bi, bj, left, solve);
             t.op = solve ? XK_OP_TRSM_DIAG : XK_OP_TRMM_DIAG;
             t.out_key = keyO;
             t.keyA = keyD;
@@ -893,7 +893,7 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
                     int keyB_ = left ? key_of(mc, q, bj) : opA(q, kx);
                     const int64_t kt = std::min(T, ka - q * T);
                     Task g;
-                    g.gpu = owner(bi, bj);
+                    g.gpu = owner_trxm(bi, bj, left, solve);
                     g.op = XK_OP_GEMM;
                     g.out_key = keyO;
                     g.keyA = keyA_;
@@ -929,7 +929,7 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
                 const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
                 const int64_t kt = std::min(T, ka - kx * T);
                 Task g;
-                g.gpu = owner(bi, bj);
+                g.gpu = owner_trxm(bi, bj, left, solve);
                 g.op = XK_OP_GEMM;
                 g.out_key = keyO;
                 g.keyA = keyA_;

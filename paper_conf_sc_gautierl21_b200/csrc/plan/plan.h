@@ -105,6 +105,18 @@ public:
         const int64_t idx = lower ? j * t - j * (j - 1) / 2 + (i - j) : j * (j + 1) / 2 + i;
         return (int)(idx % topo_.G);
     }
+    // Owner of tile (i, j) of TRMM's B (reading R12): 2D block-cyclic with the grid
+    // index along the solved dimension "snaked" (0..P-1, P-1..0, ...), so that the rows
+    // (columns) with more updates -- the work of row r grows with r -- spread evenly
+    static int64_t snake(int64_t x, int64_t n) {
+        const int64_t blk = x / n, r = x % n;
+        return (blk % 2 == 0) ? r : n - 1 - r;
+    }
+    int owner_trxm(int64_t i, int64_t j, bool left, bool solve) const {
+        if (solve) return owner(i, j);  // TRSM: the diagonal chain, not the balance, binds
+        return left ? (int)(snake(i, flags_.P) * flags_.Q + j % flags_.Q)
+                    : (int)((i % flags_.P) * flags_.Q + snake(j, flags_.Q));
+    }
     const Flags &flags() const { return flags_; }
     int64_t next_seq() const { return seq_; }  // seq of the next record to be emitted
     int link_class(int s, int d) const { return cls_[(size_t)s * (topo_.G + 1) + d]; }

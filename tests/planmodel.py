@@ -214,6 +214,16 @@ class Model:
         return out
 
     # ---- task generators: program order, symbolic versions (readings in DESIGN.md)
+    def owner_trxm(self, i, j, left, solve):
+        """TRMM's B (R12): 2D block-cyclic, grid index along the triangular
+        dimension snaked 0..P-1, P-1..0, ...; TRSM keeps the plain 2D block-cyclic map."""
+        if solve:
+            return self.owner(i, j)
+        def snake(x, n):
+            blk, r = divmod(x, n)
+            return r if blk % 2 == 0 else n - 1 - r
+        return snake(i, self.P) * self.Q + j % self.Q if left else (i % self.P) * self.Q + snake(j, self.Q)
+
     def owner_tri(self, i, j, lower, t):
         """Triangular outputs (SYRK/SYR2K, R11): the stored triangle's tiles in
         column-major order, dealt round-robin over the GPUs."""
@@ -396,7 +406,8 @@ class Model:
                 for i in range(tm):
                     ct = self.tile(C, ldc, i, j)
                     mt, nt = min(T, m - i * T), min(T, n - j * T)
-                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, [], (0, (i + j) % tmod, i, j, 0), mt * nt, -1))
+                    tasks.append(self._task(vers, OP_SCALE, i, j, ct, [], (0, (i + j) % tmod, i, j, 0), mt * nt, -1,
+                                            gpu=self.owner_trxm(i, j, left, solve)))
             return tasks
         self.matrix(A, lda, ka, ka)
 
@@ -416,7 +427,8 @@ class Model:
                 mt, nt = min(T, m - bi * T), min(T, n - bj * T)
                 fl = mt * mt * nt if left else mt * nt * nt
                 tasks.append(self._task(vers, OP_TRSM_DIAG if solve else OP_TRMM_DIAG, bi, bj, ot,
-                                        [(opA(kx, kx), 0), (ot, 2)], (s, 0, (bi + bj + s) % tmod, bi, bj), fl, s))
+                                        [(opA(kx, kx), 0), (ot, 2)], (s, 0, (bi + bj + s) % tmod, bi, bj), fl, s,
+                                        gpu=self.owner_trxm(bi, bj, left, solve)))
                 if not solve:
                     ph = 1
                     # contributions nearest the diagonal first (R9)
@@ -429,7 +441,8 @@ class Model:
                         else:
                             ins = [(self.tile(C, ldc, bi, q), 2), (opA(q, kx), 0), (ot, 2)]
                         tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins,
-                                                (s, ph, (bi + bj + s) % tmod, bi, bj), 2 * mt * nt * kt, s))
+                                                (s, ph, (bi + bj + s) % tmod, bi, bj), 2 * mt * nt * kt, s,
+                                                gpu=self.owner_trxm(bi, bj, left, solve)))
                         ph += 1
             if not solve:
                 continue
@@ -452,7 +465,7 @@ class Model:
                     u = max(s, sr - D)
                     ph = 1 if sr == s + 1 else 2
                     tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins, (u, ph, sr * tk + s, (bi + bj + s) % tmod, o),
-                                            2 * mt * nt * kt, s))
+                                            2 * mt * nt * kt, s, gpu=self.owner_trxm(bi, bj, left, solve)))
         return tasks
 
     def run(self, tasks, sync, out):
