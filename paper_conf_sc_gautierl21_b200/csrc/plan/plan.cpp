@@ -850,7 +850,7 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             for (const NodeCopy &g : e.gpu) cur = cur || (g.present && g.ver == e.ver);
             b_on_gpus = cur;
         }
-    const int64_t Dw = b_on_gpus ? nsteps : 2 * (left ? flags_.P : flags_.Q);
+    const int64_t Dw = b_on_gpus ? nsteps : 2 * (left ? std::min(flags_.P, flags_.Q) : std::max(flags_.P, flags_.Q));
     for (int64_t s = 0; s < nsteps; ++s) {
         const int64_t kx = fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
         const double a_s = solve ? ((s == 0) ? c.alpha : 1.0) : c.alpha;

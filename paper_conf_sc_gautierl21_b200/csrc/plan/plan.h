@@ -9,6 +9,7 @@
 // P:491-498; owner-computes P:384-389 on a 2D block-cyclic grid P:743-747.
 // Readings are listed in DESIGN.md.
 #pragma once
+#include <algorithm>
 #include <cstdint>
 #include <functional>
 #include <string>
@@ -105,17 +106,22 @@ public:
         const int64_t idx = lower ? j * t - j * (j - 1) / 2 + (i - j) : j * (j + 1) / 2 + i;
         return (int)(idx % topo_.G);
     }
-    // Owner of tile (i, j) of TRMM's B (reading R12): 2D block-cyclic with the grid
-    // index along the solved dimension "snaked" (0..P-1, P-1..0, ...), so that the rows
-    // (columns) with more updates -- the work of row r grows with r -- spread evenly
+    // Owner of tile (i, j) of TRSM/TRMM's B.  Reading R13: the grid's larger extent goes
+    // along the untouched dimension (columns of B for a left-side op, rows for right-side),
+    // so the tiles of the row (column) a step solves are spread over more GPUs and the
+    // chain of diagonal steps shortens.  Reading R12 (TRMM only): the grid index along the
+    // triangular dimension is snaked (0..P-1, P-1..0, ...) -- the work of B's row r grows
+    // with r -- which balances the GPUs; TRSM keeps it plain (its diagonal chain binds).
     static int64_t snake(int64_t x, int64_t n) {
         const int64_t blk = x / n, r = x % n;
         return (blk % 2 == 0) ? r : n - 1 - r;
     }
     int owner_trxm(int64_t i, int64_t j, bool left, bool solve) const {
-        if (solve) return owner(i, j);  // TRSM: the diagonal chain, not the balance, binds
-        return left ? (int)(snake(i, flags_.P) * flags_.Q + j % flags_.Q)
-                    : (int)((i % flags_.P) * flags_.Q + snake(j, flags_.Q));
+        const int64_t lo = std::min(flags_.P, flags_.Q), hi = std::max(flags_.P, flags_.Q);
+        const int64_t Pg = left ? lo : hi, Qg = left ? hi : lo;
+        const int64_t pi = (!solve && left) ? snake(i, Pg) : i % Pg;
+        const int64_t qj = (!solve && !left) ? snake(j, Qg) : j % Qg;
+        return (int)(pi * Qg + qj);
     }
     const Flags &flags() const { return flags_; }
     int64_t next_seq() const { return seq_; }  // seq of the next record to be emitted

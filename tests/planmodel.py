@@ -215,14 +215,16 @@ class Model:
 
     # ---- task generators: program order, symbolic versions (readings in DESIGN.md)
     def owner_trxm(self, i, j, left, solve):
-        """TRMM's B (R12): 2D block-cyclic, grid index along the triangular
-        dimension snaked 0..P-1, P-1..0, ...; TRSM keeps the plain 2D block-cyclic map."""
-        if solve:
-            return self.owner(i, j)
+        """TRSM/TRMM's B (R13, R12): the grid's larger extent along the untouched
+        dimension; TRMM snakes the grid index along the triangular dimension."""
         def snake(x, n):
             blk, r = divmod(x, n)
             return r if blk % 2 == 0 else n - 1 - r
-        return snake(i, self.P) * self.Q + j % self.Q if left else (i % self.P) * self.Q + snake(j, self.Q)
+        lo, hi = min(self.P, self.Q), max(self.P, self.Q)
+        Pg, Qg = (lo, hi) if left else (hi, lo)
+        pi = snake(i, Pg) if (not solve and left) else i % Pg
+        qj = snake(j, Qg) if (not solve and not left) else j % Qg
+        return pi * Qg + qj
 
     def owner_tri(self, i, j, lower, t):
         """Triangular outputs (SYRK/SYR2K, R11): the stored triangle's tiles in
@@ -418,7 +420,7 @@ class Model:
         # R10 window only when B must come from the host (some tile not current on a GPU)
         b_on_gpus = all(any(c.ver == tl.ver for c in tl.gpus.values())
                         for tl in (self.tile(C, ldc, i, j) for j in range(tn) for i in range(tm)))
-        D = tk if b_on_gpus else 2 * (self.P if left else self.Q)
+        D = tk if b_on_gpus else 2 * (min(self.P, self.Q) if left else max(self.P, self.Q))
         for s in range(tk):
             kx = s if fwd else tk - 1 - s
             for o in range(other):
