@@ -28,6 +28,9 @@ namespace xk {
 namespace {
 
 constexpr int BK = 16;
+#ifndef XK_CPF
+#define XK_CPF 0  // extra k-blocks of lead for the epilogue's C prefetch (-1 = off)
+#endif
 constexpr int BM = 64, BN = 128;   // CTA tile
 constexpr int WM = 32, WN = 32;    // warp tile
 constexpr int NWM = BM / WM, NWN = BN / WN, NWARPS = NWM * NWN;
@@ -184,6 +187,25 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
 #pragma unroll 1
     for (int kb = 0; kb < KB; ++kb) {
         const int st = kb % STAGES;
+        if (kb == KB - 2 - XK_CPF) {
+            // the epilogue's C (and deferred-beta C2) reads are cold DRAM reads: pull this
+            // warp's 32 x 32 block into L2 while the last k-blocks still run (one column of
+            // 256 bytes per lane)
+            const int64_t col = n0 + wn + lane;
+            const int64_t row = m0 + wm;
+            if (col < t.N && row < t.M) {
+                if (t.beta != 0.0) {
+                    const double *pc = t.C + row + col * t.ldc;
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(pc));
+                    if (row + 16 < t.M) asm volatile("prefetch.global.L2 [%0];" ::"l"(pc + 16));
+                }
+                if (t.beta2 != 0.0) {
+                    const double *p2 = t.C2 + row + col * t.ldc2;
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(p2));
+                    if (row + 16 < t.M) asm volatile("prefetch.global.L2 [%0];" ::"l"(p2 + 16));
+                }
+            }
+        }
 #pragma unroll
         for (int s = 0; s < BK / 4; ++s) {
             const int cur = s & 1;
