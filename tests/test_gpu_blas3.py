@@ -247,3 +247,40 @@ def test_config4_n32768_sampled(routine):
             ref = 1.5 * (L @ B0[:, j])
             bound = 4 * N * EPS * 1.5 * (np.abs(L) @ np.abs(B0[:, j]))
             assert np.all(np.abs(X[:, j] - ref) <= bound + 4 * N * EPS * np.abs(ref))
+
+
+@pytest.mark.parametrize("routine", ["dsyrk", "dsyr2k", "dtrmm", "dtrsm", "dsymm"])
+def test_owner_maps_do_not_change_bits(routine):
+    """Readings R11-R13 (triangle round-robin for SYRK/SYR2K, TRSM/TRMM grid oriented along
+    B's untouched dimension, TRMM rows snaked) only move tiles between GPUs: every tile's
+    chain of operations is the same, so 8 logical GPUs (4x2 grid) give the bits of 1 GPU --
+    on real-valued inputs, both sides / triangles."""
+    n, k, T = 300, 170, 64
+    A = inputs.uniform(1, n, n); B = inputs.uniform(2, n, n); C0 = inputs.uniform(3, n, n)
+    L = inputs.tri_dd(4, n, lower=True, fill=0.0); U = np.asfortranarray(L.T)
+    Ak = inputs.uniform(5, n, k); Bk = inputs.uniform(6, n, k)
+
+    def run(G):
+        xk.init(ngpus=G, phys=device_map(G), tile=T, probe=False)
+        outs = []
+        try:
+            for side, uplo in itertools.product("LR", "LU"):
+                X = C0.copy(order="F")
+                if routine == "dsyrk":
+                    assert xk.dsyrk(uplo, "N" if side == "L" else "T", n, k if side == "L" else n, 1.5,
+                                    Ak if side == "L" else A, n, -0.75, X, n) == 0
+                elif routine == "dsyr2k":
+                    assert xk.dsyr2k(uplo, "N", n, k, 1.5, Ak, n, Bk, n, -0.75, X, n) == 0
+                elif routine == "dsymm":
+                    assert xk.dsymm(side, uplo, n, n, 1.5, A, n, B, n, -0.75, X, n) == 0
+                else:
+                    f = xk.dtrsm if routine == "dtrsm" else xk.dtrmm
+                    tri = L if uplo == "L" else U
+                    assert f(side, uplo, "N", "N", n, n, 1.5, tri, n, X, n) == 0
+                outs.append(X)
+        finally:
+            xk.finalize()
+        return outs
+
+    for a, b in zip(run(1), run(8)):
+        assert np.array_equal(a, b)
