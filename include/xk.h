@@ -171,8 +171,10 @@ int xk_memory_coherent_sync(int64_t m, int64_t n, double *A, int64_t lda);
 int xk_memory_coherent_async(int64_t m, int64_t n, double *A, int64_t lda);
 /* Wait for all issued work.  Does NOT make host copies coherent (lazy). */
 int xk_sync(void);
-/* Drop the device copies of the tiles of a view (waits for pending work first).
- * Stale host tiles are NOT written back: call xk_memory_coherent_sync first. */
+/* Drop the device copies of the tiles of a view (waits for pending work first); from then
+ * on the host array is the valid copy of those tiles (whatever the caller holds there is
+ * read by the next call).  Stale host tiles are NOT written back: call
+ * xk_memory_coherent_sync first to keep results that live only on the GPUs. */
 int xk_memory_invalidate(int64_t m, int64_t n, const double *A, int64_t lda);
 /* Load the tiles of a host view onto their owner GPUs now (data-on-device runs). */
 int xk_memory_prefetch_async(int64_t m, int64_t n, const double *A, int64_t lda);

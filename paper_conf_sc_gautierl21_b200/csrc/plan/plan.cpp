@@ -1077,6 +1077,13 @@ void Planner::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
         if (e.bi * T >= rend || e.bi * T + e.rows <= r0) continue;
         if (e.bj * T >= cend || e.bj * T + e.cols <= c0) continue;
         for (auto &g : e.gpu) g.present = false;
+        // the host array is the valid copy from now on (drop-in semantics: whatever the
+        // caller holds there is used next; stale tiles are not written back)
+        e.host.present = true;
+        e.host.ver = e.ver;
+        e.host.t_done = 0;
+        e.host.producer = -1;
+        e.host.depth = 0;
     }
 }
 

@@ -615,3 +615,4 @@ class Model:
             if bi * T >= rend or bi * T + t.rows <= r0 or bj * T >= cend or bj * T + t.cols <= c0:
                 continue
             t.gpus = {}
+            t.host = Copy(t.ver, 0, -1, 0)  # the host array is the valid copy from now on

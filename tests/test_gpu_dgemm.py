@@ -301,3 +301,24 @@ def test_out_of_memory_fails_cleanly():
     C2 = np.zeros((N, N), order="F")
     assert xk.dgemm("N", "N", 512, 512, 512, 1.0, A, N, B, N, 0.0, C2, N) == 0
     xk.finalize()
+
+
+def test_invalidate_without_coherence_then_host_rewrite():
+    """The host array is authoritative after xk_memory_invalidate: results that lived only
+    on the GPUs are dropped, the caller rewrites the host array, and the next call reads it."""
+    N, T = 300, 128
+    A, B = inputs.integers(1, N, N), inputs.integers(2, N, N)
+    D = np.zeros((N, N), order="F")
+    logical(2, tile=T)
+    try:
+        assert xk.dgemm_async("N", "N", N, N, N, 1.0, A, N, B, N, 0.0, D, N) == 0
+        xk.sync()
+        xk.memory_invalidate(N, N, D, N)          # D's result never reaches the host
+        D[:] = inputs.integers(3, N, N)           # the caller's new contents
+        E = np.zeros((N, N), order="F")
+        assert xk.dgemm("N", "N", N, N, N, 1.0, D, N, B, N, 0.0, E, N) == 0
+    finally:
+        xk.finalize()
+    ref = np.zeros((N, N), order="F")
+    oracle.dgemm("N", "N", N, N, N, 1.0, np.asfortranarray(inputs.integers(3, N, N)), B, 0.0, ref)
+    assert np.array_equal(E, ref)

@@ -526,3 +526,19 @@ def test_trsm_window_depends_on_residency(G):
         host, _ = both(bw, flags, [trsm])
         assert update_steps(res[1]) == sorted(update_steps(res[1]))
         assert update_steps(host[0]) != sorted(update_steps(host[0]))
+
+
+def test_invalidate_makes_host_authoritative():
+    """xk_memory_invalidate drops the GPU copies and makes the host array the valid copy,
+    even when the GPUs held the only current version (no coherence first): the next call
+    reads the tiles from the host (H2D), never fails for want of a valid copy."""
+    G = 4
+    bw = TOPOS["uniform"](G)
+    flags = dict(topo="ranked", optimistic=True, window=2, tile=4)
+    calls = [gemm(m=12, n=12, k=12, C=D_ADDR, ldc=12, sync=False, beta=0.0),       # D only on GPUs
+             dict(routine=pm.INVALIDATE, m=12, n=12, C=D_ADDR, ldc=12),          # dropped, host wins
+             gemm(m=12, n=12, k=12, A=D_ADDR, lda=12, B=C_ADDR, ldb=12, C=E_ADDR, ldc=12, sync=True)]
+    got, exp = both(bw, flags, calls)
+    assert got == exp
+    d_reads = [r for r in got[2] if r[1] == pm.H2D and r[2] == 0]
+    assert len(d_reads) == 9  # every 4x4 tile of D (3 x 3 tiles) comes from the host
