@@ -677,7 +677,9 @@ int Runtime::issue(const Rec &R) {
             // diagonal solves/multiplies of one step share the diagonal tile of A: grouped
             // into one recursion over all their B tiles (grouped GEMMs, one base launch)
             if (!buf(R.keyA, g, false, &rc)) return rc;
+            if (R.keyC2 >= 0 && !buf(R.keyC2, g, false, &rc)) return rc;
             const int64_t idA = (int64_t)R.keyA * XK_MAX_GPUS + g;
+            const int64_t idC2 = R.keyC2 >= 0 ? (int64_t)R.keyC2 * XK_MAX_GPUS + g : -1;
             PendingBatch &bt = batch_[g];
             bool conflict = !bt.recs.empty() &&
                             (bt.op != R.op || bt.recs[0].keyA != R.keyA || bt.recs[0].alpha != R.alpha ||
@@ -685,13 +687,14 @@ int Runtime::issue(const Rec &R) {
                              bt.recs[0].diag != R.diag ||
                              (R.side == 'L' ? bt.recs[0].m != R.m : bt.recs[0].n != R.n));
             conflict = conflict || (int)bt.recs.size() >= max_batch_ || bt.touches(idO, true) ||
-                       bt.touches(idA, false);
+                       bt.touches(idA, false) || (idC2 >= 0 && bt.touches(idC2, false));
             for (int q = 0; q < 4 && !conflict; ++q)
                 if (r.dep[q] >= 0 && bt.contains_seq(r.dep[q])) conflict = true;
             if (conflict && (rc = flush_batch(g))) return rc;
             bt.recs.push_back(R);
             bt.out_ids.push_back(idO);
             bt.in_ids.push_back(idA);
+            if (idC2 >= 0) bt.in_ids.push_back(idC2);
             bt.op = R.op;
             return XK_OK;
         }
@@ -898,6 +901,17 @@ int Runtime::flush_batch(int g) {
         }
         cudaEvent_t ta = nullptr;
         if (tracing_ && (rc = trace_begin(g, s, &ta))) return rc;
+        // TRMM from a shadow (reading R15): the input tile is copied into the output tile,
+        // then multiplied in place with the others of the group
+        for (int q = 0; q < nb; ++q) {
+            const Rec &R = bt.recs[q];
+            if (R.keyC2 < 0) continue;
+            Buffer *S = buf(R.keyC2, g, false, &rc);
+            if (!S) return rc;
+            cudaError_t ce = cudaMemcpy2DAsync(Bp[q], (size_t)ldb[q] * 8, S->p, (size_t)S->ld * 8,
+                                               (size_t)R.m * 8, (size_t)R.n, cudaMemcpyDeviceToDevice, s);
+            if (ce != cudaSuccess) return cuda_fail(ce, "shadow tile copy");
+        }
         cudaError_t ke = launch_trxm_batch(bt.op == XK_OP_TRSM_DIAG, R0.side, R0.uplo, R0.ta, R0.diag,
                                            R0.side == 'L' ? R0.m : R0.n, R0.alpha, A->p, A->ld, nb, Bp,
                                            ldb, other, s);
@@ -914,6 +928,7 @@ int Runtime::flush_batch(int g) {
             Buffer *O = buf(R.key, g, false, &rc);
             O->writer = ev;
             O->readers.clear();
+            if (R.keyC2 >= 0) add_reader(*buf(R.keyC2, g, false, &rc), ev);
             stats.tasks[g]++;
             stats.flops[g] += R.r.work;
         }

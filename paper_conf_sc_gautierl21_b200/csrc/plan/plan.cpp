@@ -851,8 +851,20 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             b_on_gpus = cur;
         }
     const int64_t Dw = b_on_gpus ? nsteps : 2 * (left ? std::min(flags_.P, flags_.Q) : std::max(flags_.P, flags_.Q));
+    // TRMM from the host on one GPU (reading R15): every step reads B's input tiles from a
+    // per-call shadow, so no GEMM reads a tile the sweep overwrites and the sweep runs in the
+    // solve direction (top-down for left/lower): step s needs one new row (column) of B
+    // instead of the in-place order's all of B during step 0.  The diagonal multiply copies
+    // its shadow tile into the output tile first (device-to-device); B crosses PCIe once.
+    // One GPU only: with G > 1 a peer's later host read of a shadow tile could race the
+    // write-back of the output tile that shares its host memory.
+    bool sh_ok = !solve && flags_.P * flags_.Q == 1 && tk >= 2;
+    for (int64_t j = 0; j < tn && sh_ok; ++j)
+        for (int64_t i = 0; i < tm && sh_ok; ++i) sh_ok = defer_beta(key_of(mc, i, j));
+    const int ms = sh_ok ? add_shadow(mc) : -1;
+    const bool sweep_fwd = ms >= 0 ? !fwd : fwd;
     for (int64_t s = 0; s < nsteps; ++s) {
-        const int64_t kx = fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
+        const int64_t kx = sweep_fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
         const double a_s = solve ? ((s == 0) ? c.alpha : 1.0) : c.alpha;
         for (int64_t o = 0; o < other; ++o) {
             const int64_t bi = left ? kx : o, bj = left ? o : kx;
@@ -865,7 +877,13 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             t.out_key = keyO;
             t.keyA = keyD;
             t.in.push_back({keyD, V.get(keyD), 0});
-            t.in.push_back({keyO, V.get(keyO), 2});
+            if (ms >= 0) {
+                const int keyS = key_of(ms, bi, bj);
+                t.in.push_back({keyS, V.get(keyS), 2});
+                t.keyC2 = keyS;  // copied into the output tile, then multiplied in place
+            } else {
+                t.in.push_back({keyO, V.get(keyO), 2});
+            }
             t.out_ver = V.bump(keyO);
             t.ta = tA;
             t.side = left ? 'L' : 'R';
@@ -889,8 +907,9 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
                     const bool below = left ? elow : !elow;  // contributing q lie below kx
                     const int64_t q = below ? kx - dq : kx + dq;
                     if (q < 0 || q >= tk) break;
-                    int keyA_ = left ? opA(kx, q) : key_of(mc, bi, q);
-                    int keyB_ = left ? key_of(mc, q, bj) : opA(q, kx);
+                    const int mb = ms >= 0 ? ms : mc;  // B's input tiles (shadow: R15)
+                    int keyA_ = left ? opA(kx, q) : key_of(mb, bi, q);
+                    int keyB_ = left ? key_of(mb, q, bj) : opA(q, kx);
                     const int64_t kt = std::min(T, ka - q * T);
                     Task g;
                     g.gpu = owner_trxm(bi, bj, left, solve);
@@ -961,7 +980,9 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             }
         }
     }
-    return run_tasks(tasks, c.sync != 0, out, err);
+    int rc = run_tasks(tasks, c.sync != 0, out, err);
+    drop_shadow(ms);
+    return rc;
 }
 
 bool Planner::view_tiles(uint64_t base, int64_t m, int64_t n, int64_t ld, int *mat, int64_t *r0,

@@ -177,7 +177,7 @@ class Model:
                 tasks = self.gen_trxm(routine == DTRSM, left, lower, ta, diag.upper(), m, n, alpha, A, lda, C, ldc)
             if tasks:
                 self.run(tasks, sync, out)
-            if routine in (DGEMM, DSYRK, DSYR2K, DSYMM):
+            if routine in (DGEMM, DSYRK, DSYR2K, DSYMM, DTRMM):
                 self.drop_shadow(ldc)
             if sync and tasks is not None:
                 self.full_sync()
@@ -421,15 +421,24 @@ class Model:
         b_on_gpus = all(any(c.ver == tl.ver for c in tl.gpus.values())
                         for tl in (self.tile(C, ldc, i, j) for j in range(tn) for i in range(tm)))
         D = tk if b_on_gpus else 2 * (min(self.P, self.Q) if left else max(self.P, self.Q))
+        # R15: TRMM from the host on one GPU reads B's input tiles from a per-call shadow and
+        # sweeps in the solve direction; the diagonal multiply starts from the shadow tile
+        shadow = None
+        if (not solve and self.P * self.Q == 1 and tk >= 2
+                and all(self.host_only(self.tile(C, ldc, i, j)) for j in range(tn) for i in range(tm))):
+            shadow = self.new_shadow(C, ldc)
+        Bin = shadow if shadow is not None else C
+        sweep_fwd = (not fwd) if shadow is not None else fwd
         for s in range(tk):
-            kx = s if fwd else tk - 1 - s
+            kx = s if sweep_fwd else tk - 1 - s
             for o in range(other):
                 bi, bj = (kx, o) if left else (o, kx)
                 ot = self.tile(C, ldc, bi, bj)
                 mt, nt = min(T, m - bi * T), min(T, n - bj * T)
                 fl = mt * mt * nt if left else mt * nt * nt
+                src = self.tile(shadow, ldc, bi, bj) if shadow is not None else ot
                 tasks.append(self._task(vers, OP_TRSM_DIAG if solve else OP_TRMM_DIAG, bi, bj, ot,
-                                        [(opA(kx, kx), 0), (ot, 2)], (s, 0, (bi + bj + s) % tmod, bi, bj), fl, s,
+                                        [(opA(kx, kx), 0), (src, 2)], (s, 0, (bi + bj + s) % tmod, bi, bj), fl, s,
                                         gpu=self.owner_trxm(bi, bj, left, solve)))
                 if not solve:
                     ph = 1
@@ -439,9 +448,9 @@ class Model:
                     for q in qs:
                         kt = min(T, ka - q * T)
                         if left:
-                            ins = [(opA(kx, q), 0), (self.tile(C, ldc, q, bj), 2), (ot, 2)]
+                            ins = [(opA(kx, q), 0), (self.tile(Bin, ldc, q, bj), 2), (ot, 2)]
                         else:
-                            ins = [(self.tile(C, ldc, bi, q), 2), (opA(q, kx), 0), (ot, 2)]
+                            ins = [(self.tile(Bin, ldc, bi, q), 2), (opA(q, kx), 0), (ot, 2)]
                         tasks.append(self._task(vers, OP_GEMM, bi, bj, ot, ins,
                                                 (s, ph, (bi + bj + s) % tmod, bi, bj), 2 * mt * nt * kt, s,
                                                 gpu=self.owner_trxm(bi, bj, left, solve)))

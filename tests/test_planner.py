@@ -542,3 +542,33 @@ def test_invalidate_makes_host_authoritative():
     assert got == exp
     d_reads = [r for r in got[2] if r[1] == pm.H2D and r[2] == 0]
     assert len(d_reads) == 9  # every 4x4 tile of D (3 x 3 tiles) comes from the host
+
+
+def test_trmm_shadow_sweep_one_gpu():
+    """Reading R15: host-resident DTRMM on one GPU reads B's input tiles from a per-call
+    shadow and sweeps in the solve direction (top-down for left/lower, row 0 first), each
+    B tile crossing PCIe once (the shadow's H2D; the output tile gets a device copy); the
+    diagonal multiply of row kx needs only the shadow tiles of rows <= kx.  With G > 1, or
+    with B already on the GPU, the plan stays the in-place bottom-up sweep."""
+    T, t = 4, 4
+    N = T * t
+    call = xk.make_call(routine=pm.DTRMM, side="L", uplo="L", transA="N", diag="N", m=N, n=N,
+                        alpha=1.0, A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True)
+    recs = xk.plan_dump(call, uniform(1), tile=T)
+    by_seq = {r[0]: r for r in recs}
+    diag = [r for r in recs if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG]
+    assert [r[3] for r in diag] == sorted(r[3] for r in diag) and diag[0][3] == 0
+    h2d_b = [(r[3], r[4]) for r in recs if r[1] == pm.H2D and r[2] == 2]
+    assert sorted(h2d_b) == sorted(set(h2d_b)) and len(h2d_b) == t * t
+    for r in diag:  # input 1 is the shadow tile's own H2D
+        src = by_seq[r[14][1]]
+        assert src[1] == pm.H2D and (src[3], src[4]) == (r[3], r[4])
+    seen_rows = set()
+    for r in recs:
+        if r[1] == pm.H2D and r[2] == 2:
+            seen_rows.add(r[3])
+        if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG:
+            assert seen_rows <= set(range(r[3] + 1)), (r[3], seen_rows)
+    recs2 = xk.plan_dump(call, uniform(2), tile=T)
+    diag2 = [r[3] for r in recs2 if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG]
+    assert diag2[0] == t - 1 and diag2 == sorted(diag2, reverse=True)
