@@ -240,6 +240,10 @@ bool Planner::emit_copy(int key, int64_t ver, int d, int64_t treq, int operand,
     c.t_done = t1;
     c.producer = R.r.seq;
     c.depth = depth;
+    // R15: a read-once shadow's host memory is rewritten by the write-back of the output tile
+    // it shadows, so after its one host read every other copy is forwarded from a GPU (all of
+    // them descend from this H2D, which the output tile's own chain also waits on)
+    if (src == XK_HOST && mats_[e.mat].host_once) e.host.present = false;
     return true;
 }
 
@@ -851,17 +855,18 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             b_on_gpus = cur;
         }
     const int64_t Dw = b_on_gpus ? nsteps : 2 * (left ? std::min(flags_.P, flags_.Q) : std::max(flags_.P, flags_.Q));
-    // TRMM from the host on one GPU (reading R15): every step reads B's input tiles from a
+    // TRMM from the host (reading R15): every step reads B's input tiles from a
     // per-call shadow, so no GEMM reads a tile the sweep overwrites and the sweep runs in the
     // solve direction (top-down for left/lower): step s needs one new row (column) of B
     // instead of the in-place order's all of B during step 0.  The diagonal multiply copies
     // its shadow tile into the output tile first (device-to-device); B crosses PCIe once.
-    // One GPU only: with G > 1 a peer's later host read of a shadow tile could race the
-    // write-back of the output tile that shares its host memory.
-    bool sh_ok = !solve && flags_.P * flags_.Q == 1 && tk >= 2;
+    // The shadow is read from the host once per tile (host_once): a peer's later host read
+    // could otherwise race the write-back of the output tile sharing its host memory.
+    bool sh_ok = !solve && tk >= 2;
     for (int64_t j = 0; j < tn && sh_ok; ++j)
         for (int64_t i = 0; i < tm && sh_ok; ++i) sh_ok = defer_beta(key_of(mc, i, j));
     const int ms = sh_ok ? add_shadow(mc) : -1;
+    if (ms >= 0) mats_[ms].host_once = true;
     const bool sweep_fwd = ms >= 0 ? !fwd : fwd;
     for (int64_t s = 0; s < nsteps; ++s) {
         const int64_t kx = sweep_fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step

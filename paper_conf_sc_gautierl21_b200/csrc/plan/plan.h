@@ -41,6 +41,7 @@ struct Matrix {
     int64_t ld = 0;
     int64_t rows = 0, cols = 0;  // stored extent covered by the tiles known so far
     bool shadow = false;         // per-call read-only view of C's input values (beta deferral)
+    bool host_once = false;      // shadow read from the host at most once (R15: TRMM's B)
 };
 
 struct NodeCopy {

@@ -58,6 +58,7 @@ class Tile:
         self.ver = 0
         self.host = Copy(0, 0, -1, 0)  # inputs start valid on the host
         self.gpus = {}  # g -> Copy
+        self.once = False  # R15: read-once shadow
 
 
 class Model:
@@ -65,6 +66,7 @@ class Model:
                  grid=(0, 0), tile=2048):
         self.bw = [list(r) for r in bw]
         self.G = len(bw) - 1
+        self.once = set()  # read-once shadow bases (R15)
         self.cls = classes(self.bw)
         self.rate = rate_mflops
         self.mode = {"ranked": RANKED, "unranked": UNRANKED, "home": HOME}[topo] if isinstance(topo, str) else topo
@@ -89,6 +91,7 @@ class Model:
         if key not in self.tiles:
             rows, cols = self.extent[(base, ld)]
             self.tiles[key] = Tile(min(self.T, rows - bi * self.T), min(self.T, cols - bj * self.T), bi, bj)
+            self.tiles[key].once = base in self.once
         return self.tiles[key]
 
     def matrix(self, base, ld, rows, cols):
@@ -146,6 +149,8 @@ class Model:
                     state, depth, start, end, nbytes, (dep, -1, -1, -1), -1))
         t.gpus[d] = Copy(ver, end, self.seq, depth)
         self.seq += 1
+        if src == HOSTID and t.once:  # R15: later copies are forwarded from GPUs
+            t.host = None
 
     def copy_out(self, t, src, sub, ready, dep, out):
         r0, c0, rows, cols = sub
@@ -421,12 +426,13 @@ class Model:
         b_on_gpus = all(any(c.ver == tl.ver for c in tl.gpus.values())
                         for tl in (self.tile(C, ldc, i, j) for j in range(tn) for i in range(tm)))
         D = tk if b_on_gpus else 2 * (min(self.P, self.Q) if left else max(self.P, self.Q))
-        # R15: TRMM from the host on one GPU reads B's input tiles from a per-call shadow and
+        # R15: TRMM from the host reads B's input tiles from a per-call shadow and
         # sweeps in the solve direction; the diagonal multiply starts from the shadow tile
         shadow = None
-        if (not solve and self.P * self.Q == 1 and tk >= 2
+        if (not solve and tk >= 2
                 and all(self.host_only(self.tile(C, ldc, i, j)) for j in range(tn) for i in range(tm))):
             shadow = self.new_shadow(C, ldc)
+            self.once.add(shadow)  # read from the host at most once per tile
         Bin = shadow if shadow is not None else C
         sweep_fwd = (not fwd) if shadow is not None else fwd
         for s in range(tk):

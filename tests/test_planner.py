@@ -544,12 +544,11 @@ def test_invalidate_makes_host_authoritative():
     assert len(d_reads) == 9  # every 4x4 tile of D (3 x 3 tiles) comes from the host
 
 
-def test_trmm_shadow_sweep_one_gpu():
-    """Reading R15: host-resident DTRMM on one GPU reads B's input tiles from a per-call
+def test_trmm_shadow_sweep():
+    """Reading R15: host-resident DTRMM reads B's input tiles from a per-call
     shadow and sweeps in the solve direction (top-down for left/lower, row 0 first), each
     B tile crossing PCIe once (the shadow's H2D; the output tile gets a device copy); the
-    diagonal multiply of row kx needs only the shadow tiles of rows <= kx.  With G > 1, or
-    with B already on the GPU, the plan stays the in-place bottom-up sweep."""
+    diagonal multiply of row kx needs only the shadow tiles of rows <= kx."""
     T, t = 4, 4
     N = T * t
     call = xk.make_call(routine=pm.DTRMM, side="L", uplo="L", transA="N", diag="N", m=N, n=N,
@@ -569,6 +568,16 @@ def test_trmm_shadow_sweep_one_gpu():
             seen_rows.add(r[3])
         if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG:
             assert seen_rows <= set(range(r[3] + 1)), (r[3], seen_rows)
-    recs2 = xk.plan_dump(call, uniform(2), tile=T)
-    diag2 = [r[3] for r in recs2 if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG]
-    assert diag2[0] == t - 1 and diag2 == sorted(diag2, reverse=True)
+    # G > 1: the same sweep; every shadow tile is read from the host at most once in every
+    # source mode (later copies are forwarded), so no host read can follow the write-back of
+    # the output tile that shares its host memory
+    for G in (2, 4, 8):
+        for mode, opt in (("ranked", True), ("ranked", False), ("home", False)):
+            recs2 = xk.plan_dump(call, uniform(G), tile=T, topo=mode, optimistic=opt)
+            diag2 = [r[3] for r in recs2 if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG]
+            assert diag2[0] == 0 and sorted(diag2) == sorted(r for r in range(t) for _ in range(t))
+            h2d = [(r[3], r[4]) for r in recs2 if r[1] == pm.H2D and r[2] == 2]
+            assert sorted(h2d) == sorted(set(h2d)) and len(h2d) == t * t, (G, mode)
+            d2h_seq = {(r[3], r[4]): r[0] for r in recs2 if r[1] == pm.D2H}
+            h2d_seq = {(r[3], r[4]): r[0] for r in recs2 if r[1] == pm.H2D and r[2] == 2}
+            assert all(h2d_seq[k] < d2h_seq[k] for k in d2h_seq)

@@ -31,7 +31,7 @@ REPS = int(os.environ.get("REPS", 3))
 R = os.environ.get("ROUTINE", "dgemm")
 MODES = [("full", "ranked", True), ("no_opt", "ranked", False), ("no_opt_topo", "unranked", False),
          ("home", "home", True), ("dod", "ranked", True)]
-FLOPS = {"dgemm": 2.0 * N ** 3, "dsyr2k": 2.0 * N ** 3 + N, "dtrsm": 1.0 * N ** 3}[R]
+FLOPS = {"dgemm": 2.0 * N ** 3, "dsyr2k": 2.0 * N ** 3 + N, "dtrsm": 1.0 * N ** 3, "dtrmm": 1.0 * N ** 3}[R]
 
 A = inputs.uniform(1, N, N)
 B = inputs.uniform(2, N, N)
@@ -44,6 +44,8 @@ def call(asynchronous=False):
         return (xk.dgemm_async if asynchronous else xk.dgemm)("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
     if R == "dsyr2k":
         return xk.dsyr2k("L", "N", N, N, 1.5, A, N, B, N, -0.75, C, N, asynchronous=asynchronous)
+    if R == "dtrmm":
+        return xk.dtrmm("L", "L", "N", "N", N, N, 1.0, L, N, B, N, asynchronous=asynchronous)
     return xk.dtrsm("L", "L", "N", "N", N, N, 1.0, L, N, B, N, asynchronous=asynchronous)
 
 
