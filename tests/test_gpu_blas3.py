@@ -284,3 +284,38 @@ def test_owner_maps_do_not_change_bits(routine):
 
     for a, b in zip(run(1), run(8)):
         assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("G", [1, 8])
+def test_trmm_shadow_matches_in_place(G):
+    """Reading R15: host-resident DTRMM runs the shadow sweep (B's input from a per-call
+    shadow, top-down), data-on-device DTRMM the in-place bottom-up sweep.  Each output tile
+    sums the same terms in the same order (diagonal multiply, then contributions nearest the
+    diagonal first), so the two results are bitwise equal; and the shadow sweep moves B over
+    PCIe exactly once (H2D = B + the stored triangle's tiles of A)."""
+    T = 128
+    xk.init(ngpus=G, phys=device_map(G), tile=T, probe=False)
+    try:
+        m, n = 300, 260
+        L = inputs.tri_dd(4, m, lower=True, fill=np.nan)
+        B0 = inputs.uniform(2, m, n)
+        X1 = B0.copy(order="F")
+        xk.reset_stats()
+        assert xk.dtrmm("L", "L", "N", "N", m, n, 1.5, L, m, X1, m) == 0
+        st = xk.get_stats()
+        rows = [min(T, m - i * T) for i in range(-(-m // T))]
+        tri_bytes = 8 * sum(rows[i] * rows[j] for i in range(len(rows)) for j in range(i + 1))
+        assert sum(st["h2d_bytes"]) == 8 * m * n + tri_bytes
+        X2 = B0.copy(order="F")
+        xk.memory_prefetch_async(m, n, X2, m)
+        xk.memory_prefetch_async(m, m, L, m)
+        xk.sync()
+        assert xk.dtrmm("L", "L", "N", "N", m, n, 1.5, L, m, X2, m, asynchronous=True) == 0
+        assert xk.memory_coherent_sync(m, n, X2, m) == 0
+        assert np.array_equal(X1, X2)
+        ref = B0.copy(order="F")
+        oracle.dtrmm("L", "L", "N", "N", m, n, 1.5, L, ref)
+        T_ = tri_of(L, True, False)
+        assert np.all(np.abs(X1 - ref) <= 4 * m * EPS * 1.5 * (np.abs(T_) @ np.abs(B0)))
+    finally:
+        xk.finalize()
