@@ -1113,8 +1113,31 @@ void Planner::invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld) {
     }
 }
 
+// Drop the GPU copies of a view's tiles whose host copy is current.  A tile whose only
+// current copy is on a GPU (the output of an earlier async call, not yet made coherent) is
+// kept as it is: dropping it would lose the result (xk_memory_coherent_sync writes it back
+// later), and marking the stale host data valid would hand it to the next reader.
+void Planner::release(uint64_t base, int64_t m, int64_t n, int64_t ld) {
+    int mat;
+    int64_t r0, c0;
+    if (m <= 0 || n <= 0) return;
+    if (!view_tiles(base, m, n, ld, &mat, &r0, &c0)) return;
+    const int64_t T = flags_.T;
+    const Matrix &M = mats_[mat];
+    int64_t rend = std::min(M.rows, r0 + m), cend = std::min(M.cols, c0 + n);
+    for (auto &kv : keymap_) {
+        Entry &e = entries_[kv.second];
+        if (e.mat != mat) continue;
+        if (e.bi * T >= rend || e.bi * T + e.rows <= r0) continue;
+        if (e.bj * T >= cend || e.bj * T + e.cols <= c0) continue;
+        if (!(e.host.present && e.host.ver == e.ver)) continue;  // GPU-dirty: keep
+        for (auto &g : e.gpu) g.present = false;
+    }
+}
+
 // After a synchronous routine: a full sync point, then the operands' device copies are
-// dropped (sync routines are drop-in).
+// dropped (sync routines are drop-in) -- except those of tiles whose current
+// version exists only on a GPU (see release()).
 void Planner::finish_call(const xk_call_t &c) {
     full_sync();
     const bool ta = is_t(c.transA), tb = is_t(c.transB);
@@ -1122,32 +1145,32 @@ void Planner::finish_call(const xk_call_t &c) {
     switch (c.routine) {
     case XK_ROUTINE_DGEMM:
         if (c.alpha != 0.0 && c.k > 0) {
-            invalidate(c.A, ta ? c.k : c.m, ta ? c.m : c.k, (int64_t)c.lda);
-            invalidate(c.B, tb ? c.n : c.k, tb ? c.k : c.n, (int64_t)c.ldb);
+            release(c.A, ta ? c.k : c.m, ta ? c.m : c.k, (int64_t)c.lda);
+            release(c.B, tb ? c.n : c.k, tb ? c.k : c.n, (int64_t)c.ldb);
         }
-        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        release(c.C, c.m, c.n, (int64_t)c.ldc);
         break;
     case XK_ROUTINE_DSYRK:
     case XK_ROUTINE_DSYR2K:
         if (c.alpha != 0.0 && c.k > 0) {
-            invalidate(c.A, ta ? c.k : c.n, ta ? c.n : c.k, (int64_t)c.lda);
+            release(c.A, ta ? c.k : c.n, ta ? c.n : c.k, (int64_t)c.lda);
             if (c.routine == XK_ROUTINE_DSYR2K)
-                invalidate(c.B, ta ? c.k : c.n, ta ? c.n : c.k, (int64_t)c.ldb);
+                release(c.B, ta ? c.k : c.n, ta ? c.n : c.k, (int64_t)c.ldb);
         }
-        invalidate(c.C, c.n, c.n, (int64_t)c.ldc);
+        release(c.C, c.n, c.n, (int64_t)c.ldc);
         break;
     case XK_ROUTINE_DSYMM:
         if (c.alpha != 0.0) {
             const int64_t ka = left ? c.m : c.n;
-            invalidate(c.A, ka, ka, (int64_t)c.lda);
-            invalidate(c.B, c.m, c.n, (int64_t)c.ldb);
+            release(c.A, ka, ka, (int64_t)c.lda);
+            release(c.B, c.m, c.n, (int64_t)c.ldb);
         }
-        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        release(c.C, c.m, c.n, (int64_t)c.ldc);
         break;
     default: {  // TRMM / TRSM
         const int64_t ka = left ? c.m : c.n;
-        if (c.alpha != 0.0) invalidate(c.A, ka, ka, (int64_t)c.lda);
-        invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
+        if (c.alpha != 0.0) release(c.A, ka, ka, (int64_t)c.lda);
+        release(c.C, c.m, c.n, (int64_t)c.ldc);
     }
     }
 }

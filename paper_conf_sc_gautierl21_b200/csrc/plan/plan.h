@@ -94,6 +94,8 @@ public:
     void full_sync();
     // Drop GPU copies of the tiles intersecting a view.
     void invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld);
+    // Drop the GPU copies of a view's tiles whose host copy is current (end of a sync call).
+    void release(uint64_t base, int64_t m, int64_t n, int64_t ld);
 
     const Entry &entry(int id) const { return entries_[id]; }
     const Matrix &matrix(int id) const { return mats_[id]; }

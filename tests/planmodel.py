@@ -188,26 +188,26 @@ class Model:
                 self.full_sync()
                 if routine == DGEMM:
                     if alpha != 0 and k > 0:
-                        self.invalidate(A, (k, m) if ta else (m, k), lda)
-                        self.invalidate(B, (n, k) if tb else (k, n), ldb)
-                    self.invalidate(C, (m, n), ldc)
+                        self.release(A, (k, m) if ta else (m, k), lda)
+                        self.release(B, (n, k) if tb else (k, n), ldb)
+                    self.release(C, (m, n), ldc)
                 elif routine in (DSYRK, DSYR2K):
                     if alpha != 0 and k > 0:
-                        self.invalidate(A, (k, n) if ta else (n, k), lda)
+                        self.release(A, (k, n) if ta else (n, k), lda)
                         if routine == DSYR2K:
-                            self.invalidate(B, (k, n) if ta else (n, k), ldb)
-                    self.invalidate(C, (n, n), ldc)
+                            self.release(B, (k, n) if ta else (n, k), ldb)
+                    self.release(C, (n, n), ldc)
                 elif routine == DSYMM:
                     if alpha != 0:
                         ka = m if left else n
-                        self.invalidate(A, (ka, ka), lda)
-                        self.invalidate(B, (m, n), ldb)
-                    self.invalidate(C, (m, n), ldc)
+                        self.release(A, (ka, ka), lda)
+                        self.release(B, (m, n), ldb)
+                    self.release(C, (m, n), ldc)
                 else:
                     ka = m if left else n
                     if alpha != 0:
-                        self.invalidate(A, (ka, ka), lda)
-                    self.invalidate(C, (m, n), ldc)
+                        self.release(A, (ka, ka), lda)
+                    self.release(C, (m, n), ldc)
         elif routine == COHERENT:
             self.coherent(C, m, n, ldc, out)
         elif routine == SYNC:
@@ -631,3 +631,23 @@ class Model:
                 continue
             t.gpus = {}
             t.host = Copy(t.ver, 0, -1, 0)  # the host array is the valid copy from now on
+
+    def release(self, base, shape, ld):
+        """End of a sync call: drop the GPU copies of the view's tiles whose host copy is
+        current; a tile valid only on a GPU (an earlier async call's output) keeps them."""
+        m, n = shape
+        if m <= 0 or n <= 0:
+            return
+        loc = self.locate(base, ld)
+        if loc is None:
+            return
+        b, r0, c0, rows, cols = loc
+        T = self.T
+        rend, cend = min(rows, r0 + m), min(cols, c0 + n)
+        for (bb, l, bi, bj), t in self.tiles.items():
+            if (bb, l) != (b, ld):
+                continue
+            if bi * T >= rend or bi * T + t.rows <= r0 or bj * T >= cend or bj * T + t.cols <= c0:
+                continue
+            if t.host is not None and t.host.ver == t.ver:
+                t.gpus = {}

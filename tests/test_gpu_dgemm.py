@@ -322,3 +322,43 @@ def test_invalidate_without_coherence_then_host_rewrite():
     ref = np.zeros((N, N), order="F")
     oracle.dgemm("N", "N", N, N, N, 1.0, np.asfortranarray(inputs.integers(3, N, N)), B, 0.0, ref)
     assert np.array_equal(E, ref)
+
+
+@pytest.mark.parametrize("G", [1, 4])
+def test_async_then_sync_then_coherent(G):
+    """async D = A*B, then a synchronous E = D*C2 that reads D from the
+    GPUs, then coherent(D): D comes back exactly (exact integers, bitwise vs the oracle) --
+    the sync call must not drop D's only current copies.  Also async TRSM then sync GEMM."""
+    N, T = 384, 128
+    A, B, C2 = inputs.integers(1, N, N), inputs.integers(2, N, N), inputs.integers(6, N, N)
+    ref_D = np.zeros((N, N), order="F")
+    oracle.dgemm("N", "N", N, N, N, 1.0, A, B, 0.0, ref_D)
+    ref_E = np.zeros((N, N), order="F")
+    oracle.dgemm("N", "N", N, N, N, 1.0, ref_D, C2, 0.0, ref_E)
+    logical(G, tile=T)
+    try:
+        D = np.full((N, N), -7.0, order="F")
+        E = np.full((N, N), -7.0, order="F")
+        assert xk.dgemm_async("N", "N", N, N, N, 1.0, A, N, B, N, 0.0, D, N) == 0
+        assert xk.dgemm("N", "N", N, N, N, 1.0, D, N, C2, N, 0.0, E, N) == 0
+        assert np.array_equal(E, ref_E)
+        assert np.all(D == -7.0)  # not coherent yet (lazy)
+        assert xk.memory_coherent_sync(N, N, D, N) == 0
+        assert np.array_equal(D, ref_D)
+        # TRSM (async) -> GEMM (sync) -> coherent(X): L diagonally dominant, Q13 bound on X
+        L = inputs.tri_dd(4, N, lower=True)
+        X = inputs.uniform(2, N, N)
+        X0 = X.copy(order="F")
+        F2 = np.zeros((N, N), order="F")
+        assert xk.dtrsm("L", "L", "N", "N", N, N, 1.5, L, N, X, N, asynchronous=True) == 0
+        assert xk.dgemm("N", "N", N, N, N, 1.0, X, N, C2, N, 0.0, F2, N) == 0
+        assert np.array_equal(X, X0)
+        assert xk.memory_coherent_sync(N, N, X, N) == 0
+    finally:
+        xk.finalize()
+    refX = X0.copy(order="F")
+    oracle.dtrsm("L", "L", "N", "N", N, N, 1.5, L, refX)
+    assert np.linalg.norm(X - refX) <= 1e-13 * np.linalg.norm(refX)
+    refF = np.zeros((N, N), order="F")
+    oracle.dgemm("N", "N", N, N, N, 1.0, X, C2, 0.0, refF)
+    check_bound("N", "N", N, N, N, 1.0, X, C2, 0.0, refF, F2, refF)

@@ -581,3 +581,45 @@ def test_trmm_shadow_sweep():
             d2h_seq = {(r[3], r[4]): r[0] for r in recs2 if r[1] == pm.D2H}
             h2d_seq = {(r[3], r[4]): r[0] for r in recs2 if r[1] == pm.H2D and r[2] == 2}
             assert all(h2d_seq[k] < d2h_seq[k] for k in d2h_seq)
+
+
+@pytest.mark.parametrize("G", [1, 4])
+@pytest.mark.parametrize("second", ["gemm", "trsm_then_gemm"])
+def test_sync_call_keeps_gpu_dirty_inputs(G, second):
+    """a synchronous call that reads a tile whose only current copy is on a
+    GPU (an earlier async call's output) must not drop it: a later coherent_sync of that view
+    writes every one of its tiles back, from the GPU that holds it.  Checked on the planner
+    alone (not via the mirrored model): async D = A*B (or async X = TRSM), sync E = D*C,
+    coherent(D) -> one D2H per tile of D, each after D's own last task."""
+    T, t = 4, 3
+    N = T * t
+    s = xk.PlanSession(uniform(G), topo="ranked", optimistic=True, tile=T)
+    if second == "gemm":
+        first = s.call(xk.make_call(m=N, n=N, k=N, alpha=1.0, beta=0.0, A=A_ADDR, lda=N, B=B_ADDR,
+                                    ldb=N, C=D_ADDR, ldc=N, sync=False))
+    else:
+        first = s.call(xk.make_call(routine=pm.DTRSM, side="L", uplo="L", transA="N", diag="N", m=N,
+                                    n=N, alpha=1.0, A=A_ADDR, lda=N, C=D_ADDR, ldc=N, sync=False))
+    last_task = {}
+    for r in first:
+        if r[1] == pm.TASK:
+            last_task[(r[3], r[4])] = r[0]
+    mid = s.call(xk.make_call(m=N, n=N, k=N, alpha=1.0, beta=0.0, A=D_ADDR, lda=N, B=C_ADDR, ldb=N,
+                              C=E_ADDR, ldc=N, sync=True))
+    assert not any(r[1] == pm.H2D and r[2] == 0 for r in mid)  # D read from the GPUs
+    wb = s.call(xk.make_call(routine=pm.COHERENT, m=N, n=N, C=D_ADDR, ldc=N))
+    d2h = [r for r in wb if r[1] == pm.D2H]
+    assert sorted((r[3], r[4]) for r in d2h) == [(i, j) for i in range(t) for j in range(t)]
+    for r in d2h:
+        assert r[14][0] == -1 or r[14][0] == last_task[(r[3], r[4])]
+    # a second coherent call has nothing left to write back; the next read of D is from
+    # the host only if nothing on the GPUs is current any more (the GPU copies were kept)
+    assert not [r for r in s.call(xk.make_call(routine=pm.COHERENT, m=N, n=N, C=D_ADDR, ldc=N))
+                if r[1] == pm.D2H]
+    s.close()
+    # the mirrored model agrees record for record
+    calls = [gemm(m=N, n=N, k=N, A=A_ADDR, lda=N, B=B_ADDR, ldb=N, C=D_ADDR, ldc=N, sync=False, beta=0.0),
+             gemm(m=N, n=N, k=N, A=D_ADDR, lda=N, B=C_ADDR, ldb=N, C=E_ADDR, ldc=N, sync=True, beta=0.0),
+             dict(routine=pm.COHERENT, m=N, n=N, C=D_ADDR, ldc=N)]
+    got, exp = both(uniform(G), dict(topo="ranked", optimistic=True, window=2, tile=T), calls)
+    assert got == exp
