@@ -101,6 +101,9 @@ typedef struct xk_config {
     char session[128];    /* rank mode: path of the shared control file, unique per session
                              (e.g. "/dev/shm/xk_<token>"); rank 0 creates it, rank 0 removes
                              it at xk_finalize */
+    int64_t mem_bytes;    /* tile-cache capacity per logical GPU the planner plans against
+                             (xk_flags_t.mem_bytes); 0 = derived at init: 90% of the device's
+                             free memory / logical GPUs sharing it (rank mode: the arena) */
 } xk_config_t;
 
 /* Fill *cfg with defaults, then apply the environment (XK_NGPUS, XK_TILE,
@@ -251,6 +254,9 @@ typedef struct xk_flags {
     int topo, optimistic, window;
     int grid_p, grid_q;
     int64_t tile;
+    int64_t mem_bytes; /* device tile-cache capacity per GPU the plan must fit: a per-call
+                          shadow (beta deferral Q12'', TRMM R15) is used only when every GPU's
+                          resident tiles plus the call's tiles fit; 0 = unlimited */
 } xk_flags_t;
 
 /* Tile-task operations (TASK records, field op). */

@@ -58,7 +58,8 @@ def _c(ch):
 
 # ---------------------------------------------------------------------------- lifecycle
 def init(ngpus=0, tile=0, topo=None, optimistic=None, window=0, kstreams=0, probe=None,
-         grid=None, phys=None, task_rate_mflops=0, rank=None, world=None, session=None, arena_bytes=0):
+         grid=None, phys=None, task_rate_mflops=0, rank=None, world=None, session=None, arena_bytes=0,
+         mem_bytes=0):
     """xk_init.  `phys` maps logical GPUs to physical devices (logical-device mode).
 
     Rank mode (one process per GPU): every one of `world` processes calls
@@ -96,6 +97,8 @@ def init(ngpus=0, tile=0, topo=None, optimistic=None, window=0, kstreams=0, prob
             cfg.map_devices = 1
     if arena_bytes:
         cfg.arena_bytes = int(arena_bytes)
+    if mem_bytes:
+        cfg.mem_bytes = int(mem_bytes)
     return _check(lib().xk_init(ctypes.byref(cfg)))
 
 
@@ -247,8 +250,9 @@ def _topo(bw, rate_mflops):
     return t
 
 
-def _flags(topo="ranked", optimistic=True, window=2, grid=(0, 0), tile=2048):
+def _flags(topo="ranked", optimistic=True, window=2, grid=(0, 0), tile=2048, mem_bytes=0):
     f = _abi.Flags()
+    f.mem_bytes = int(mem_bytes)
     f.topo = TOPO_NAMES[topo] if isinstance(topo, str) else int(topo)
     f.optimistic = int(bool(optimistic))
     f.window = window

@@ -38,7 +38,7 @@ class Config(ctypes.Structure):
                 ("grid_p", c_int), ("grid_q", c_int), ("tile", i64), ("topo", c_int),
                 ("optimistic", c_int), ("window", c_int), ("kstreams", c_int), ("probe", c_int),
                 ("task_rate_mflops", i64), ("rank", c_int), ("world", c_int), ("arena_bytes", i64),
-                ("session", ctypes.c_char * 128)]
+                ("session", ctypes.c_char * 128), ("mem_bytes", i64)]
 
 
 class Stats(ctypes.Structure):
@@ -59,7 +59,7 @@ class Topo(ctypes.Structure):
 
 class Flags(ctypes.Structure):
     _fields_ = [("topo", c_int), ("optimistic", c_int), ("window", c_int), ("grid_p", c_int),
-                ("grid_q", c_int), ("tile", i64)]
+                ("grid_q", c_int), ("tile", i64), ("mem_bytes", i64)]
 
 
 class Call(ctypes.Structure):

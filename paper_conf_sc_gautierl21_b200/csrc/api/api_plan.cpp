@@ -54,6 +54,7 @@ bool make_flags(const xk_flags_t *f, int G, Flags *out, std::string &err) {
         F.T = f->tile > 0 ? f->tile : 2048;
         F.P = f->grid_p;
         F.Q = f->grid_q;
+        F.mem_bytes = f->mem_bytes > 0 ? f->mem_bytes : 0;
     }
     if (F.topo < XK_TOPO_RANKED || F.topo > XK_TOPO_HOME) {
         err = "flags: unknown topo mode";

@@ -174,6 +174,24 @@ int Runtime::init(const xk_config_t &cfg) {
             return rc;
         }
     }
+    // tile-cache capacity the planner plans against (shadow plans only when they fit)
+    if (cfg.mem_bytes > 0) {
+        flags_.mem_bytes = cfg.mem_bytes;
+    } else if (rank_mode_) {
+        flags_.mem_bytes = devs_[rank_].arena_bytes;  // the same on every rank
+    } else {
+        int64_t cap = INT64_MAX;
+        for (int g = 0; g < G; ++g) {
+            int share = 0;
+            for (int h = 0; h < G; ++h) share += devs_[h].phys == devs_[g].phys;
+            size_t fr = 0, tot = 0;
+            XK_CK(cudaSetDevice(devs_[g].phys));
+            XK_CK(cudaMemGetInfo(&fr, &tot));
+            cap = std::min(cap, (int64_t)((double)fr * 0.9) / share);
+        }
+        cur_dev_ = -1;
+        flags_.mem_bytes = cap;
+    }
     planner_.reset(new Planner(topo, flags_));
     std::memset(&stats, 0, sizeof(stats));
     stats.ngpus = G;
@@ -307,7 +325,8 @@ int Runtime::init_rank_mode(const xk_config_t &cfg) {
     // plans (FNV-1a over the fields; kstreams and the like only change local issue)
     uint64_t hcfg = 1469598103934665603ull;
     for (int64_t v : {(int64_t)cfg.tile, (int64_t)cfg.topo, (int64_t)cfg.optimistic, (int64_t)cfg.window,
-                      (int64_t)cfg.grid_p, (int64_t)cfg.grid_q, (int64_t)cfg.probe, cfg.task_rate_mflops}) {
+                      (int64_t)cfg.grid_p, (int64_t)cfg.grid_q, (int64_t)cfg.probe, cfg.task_rate_mflops,
+                      cfg.mem_bytes}) {
         hcfg ^= (uint64_t)v;
         hcfg *= 1099511628211ull;
     }

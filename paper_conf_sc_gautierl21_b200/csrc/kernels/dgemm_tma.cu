@@ -215,9 +215,16 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
                     // this warp's last read of the stage is done; the last warp to get here
                     // refills the stage with block kb + STAGES (no CTA-wide barrier, no
                     // dedicated producer warp)
+                    // The count is an acq_rel RMW: each warp's increment releases its reads
+                    // of the stage (ordered before lane 0's RMW by __syncwarp), and the last
+                    // increment acquires all of them (one release sequence), so the refill's
+                    // async-proxy TMA write (after fence.proxy.async) follows every read.
                     __syncwarp();
                     if (lane == 0) {
-                        if (atomicAdd(&done_cnt[st], 1) == NWARPS - 1) {
+                        uint32_t old;
+                        asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;\n"
+                                     : "=r"(old) : "r"(smem_u32(&done_cnt[st])) : "memory");
+                        if (old == NWARPS - 1) {
                             atomicExch(&done_cnt[st], 0);
                             if (kb + STAGES < KB) {
                                 asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");

@@ -496,6 +496,33 @@ void Planner::drop_shadow(int ms) {
     mats_[ms].ld = -1;
 }
 
+// A shadow adds a second copy of C's (TRMM: B's) tiles to the device footprint, and there is
+// no eviction: the shadow plan is used only if, on every GPU, the tiles resident now plus the
+// tiles this call's tasks read or write there fit in the capacity (device buffers hold
+// round_up(rows, 16) x cols doubles).  Otherwise the call is planned without a shadow.
+bool Planner::fits(const std::vector<Task> &tasks) const {
+    if (flags_.mem_bytes <= 0) return true;
+    const int G = topo_.G;
+    std::vector<int64_t> bytes(G, 0);
+    std::vector<std::vector<char>> seen(G, std::vector<char>(entries_.size(), 0));
+    auto add = [&](int g, int key) {
+        if (key < 0 || seen[g][key]) return;
+        seen[g][key] = 1;
+        const Entry &e = entries_[key];
+        bytes[g] += 8 * ((e.rows + 15) / 16 * 16) * e.cols;
+    };
+    for (const auto &kv : keymap_)
+        for (int g = 0; g < G; ++g)
+            if (entries_[kv.second].gpu[g].present) add(g, kv.second);
+    for (const Task &t : tasks) {
+        add(t.gpu, t.out_key);
+        for (const Input &in : t.in) add(t.gpu, in.key);
+    }
+    for (int g = 0; g < G; ++g)
+        if (bytes[g] > flags_.mem_bytes) return false;
+    return true;
+}
+
 // DGEMM (PLASMA pdgemm structure): C(i,j) k-chains, beta on the first task.
 int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err) {
     const int64_t m = c.m, n = c.n, k = c.k, T = flags_.T;
@@ -513,69 +540,78 @@ int Planner::plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
     }
     const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tkn = scale_only ? 0 : cdiv(k, T);
     const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
-    const int ms = (!scale_only && c.beta != 0.0 && tkn >= 2) ? add_shadow(mc) : -1;
-    Versions V;
-    V.e = &entries_;
+    int ms = (!scale_only && c.beta != 0.0 && tkn >= 2) ? add_shadow(mc) : -1;
     std::vector<Task> tasks;
-    tasks.reserve((size_t)(tm * tn * std::max<int64_t>(tkn, 1)));
-    for (int64_t j = 0; j < tn; ++j) {
-        for (int64_t i = 0; i < tm; ++i) {
-            int keyC = key_of(mc, i, j);
-            int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
-            if (scale_only) {
-                Task t;
-                t.gpu = owner(i, j);
-                t.op = XK_OP_SCALE;
-                t.out_key = keyC;
-                if (c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
-                t.out_ver = V.bump(keyC);
-                t.beta = c.beta;
-                t.tk = -1;
-                t.i = i; t.j = j;
-                t.m = mt; t.n = nt; t.k = 0;
-                t.flops = mt * nt;
-                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
-                std::copy(sk, sk + 5, t.skey);
-                tasks.push_back(t);
-                continue;
-            }
-            const bool defer = ms >= 0 && defer_beta(keyC);
-            const int keyS = defer ? key_of(ms, i, j) : -1;
-            for (int64_t kk = 0; kk < tkn; ++kk) {
-                int64_t kt = std::min(T, k - kk * T);
-                int keyA = ta ? key_of(ma, kk, i) : key_of(ma, i, kk);
-                int keyB = tb ? key_of(mb, j, kk) : key_of(mb, kk, j);
-                Task t;
-                t.gpu = owner(i, j);
-                t.op = XK_OP_GEMM;
-                t.out_key = keyC;
-                t.in.push_back({keyA, V.get(keyA), 0});
-                t.in.push_back({keyB, V.get(keyB), 1});
-                if (kk > 0 || (c.beta != 0.0 && !defer)) t.in.push_back({keyC, V.get(keyC), 2});
-                if (defer && kk == tkn - 1) {
-                    t.in.push_back({keyS, V.get(keyS), 2});
-                    t.keyC2 = keyS;
-                    t.beta2 = c.beta;
+    for (;;) {  // with the shadow if it fits (fits()), else without
+        Versions V;
+        V.e = &entries_;
+        tasks.clear();
+        tasks.reserve((size_t)(tm * tn * std::max<int64_t>(tkn, 1)));
+        for (int64_t j = 0; j < tn; ++j) {
+            for (int64_t i = 0; i < tm; ++i) {
+                int keyC = key_of(mc, i, j);
+                int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
+                if (scale_only) {
+                    Task t;
+                    t.gpu = owner(i, j);
+                    t.op = XK_OP_SCALE;
+                    t.out_key = keyC;
+                    if (c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                    t.out_ver = V.bump(keyC);
+                    t.beta = c.beta;
+                    t.tk = -1;
+                    t.i = i; t.j = j;
+                    t.m = mt; t.n = nt; t.k = 0;
+                    t.flops = mt * nt;
+                    int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
+                    std::copy(sk, sk + 5, t.skey);
+                    tasks.push_back(t);
+                    continue;
                 }
-                t.out_ver = V.bump(keyC);
-                t.keyA = keyA;
-                t.keyB = keyB;
-                t.ta = ta ? 'T' : 'N';
-                t.tb = tb ? 'T' : 'N';
-                t.alpha = c.alpha;
-                t.beta = (kk == 0) ? (defer ? 0.0 : c.beta) : 1.0;
-                t.tk = kk;
-                t.i = i; t.j = j;
-                t.m = mt; t.n = nt; t.k = kt;
-                t.flops = 2 * mt * nt * kt;
-                // staggered k-chains (reading Q12'): tile (i,j) starts its chain at slot
-                // (i+j) mod tk, so chains begin and end at different times and C's D2H
-                // spreads over the last tk slots instead of piling up at the end
-                int64_t sk[5] = {kk + (i + j) % tkn, (i + j + kk) % tmod, i, j, 0};
-                std::copy(sk, sk + 5, t.skey);
-                tasks.push_back(t);
+                const bool defer = ms >= 0 && defer_beta(keyC);
+                const int keyS = defer ? key_of(ms, i, j) : -1;
+                for (int64_t kk = 0; kk < tkn; ++kk) {
+                    int64_t kt = std::min(T, k - kk * T);
+                    int keyA = ta ? key_of(ma, kk, i) : key_of(ma, i, kk);
+                    int keyB = tb ? key_of(mb, j, kk) : key_of(mb, kk, j);
+                    Task t;
+                    t.gpu = owner(i, j);
+                    t.op = XK_OP_GEMM;
+                    t.out_key = keyC;
+                    t.in.push_back({keyA, V.get(keyA), 0});
+                    t.in.push_back({keyB, V.get(keyB), 1});
+                    if (kk > 0 || (c.beta != 0.0 && !defer)) t.in.push_back({keyC, V.get(keyC), 2});
+                    if (defer && kk == tkn - 1) {
+                        t.in.push_back({keyS, V.get(keyS), 2});
+                        t.keyC2 = keyS;
+                        t.beta2 = c.beta;
+                    }
+                    t.out_ver = V.bump(keyC);
+                    t.keyA = keyA;
+                    t.keyB = keyB;
+                    t.ta = ta ? 'T' : 'N';
+                    t.tb = tb ? 'T' : 'N';
+                    t.alpha = c.alpha;
+                    t.beta = (kk == 0) ? (defer ? 0.0 : c.beta) : 1.0;
+                    t.tk = kk;
+                    t.i = i; t.j = j;
+                    t.m = mt; t.n = nt; t.k = kt;
+                    t.flops = 2 * mt * nt * kt;
+                    // staggered k-chains (reading Q12'): tile (i,j) starts its chain at slot
+                    // (i+j) mod tk, so chains begin and end at different times and C's D2H
+                    // spreads over the last tk slots instead of piling up at the end
+                    int64_t sk[5] = {kk + (i + j) % tkn, (i + j + kk) % tmod, i, j, 0};
+                    std::copy(sk, sk + 5, t.skey);
+                    tasks.push_back(t);
+                }
             }
         }
+        if (ms >= 0 && !fits(tasks)) {
+            drop_shadow(ms);
+            ms = -1;
+            continue;
+        }
+        break;
     }
     int rc = run_tasks(tasks, c.sync != 0, out, err);
     drop_shadow(ms);
@@ -606,80 +642,89 @@ int Planner::plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std:
     const int64_t tmod = std::max<int64_t>(1, tn);
     const int tri = lower ? 1 : 2;
     const int64_t nchain = tkn * (two ? 2 : 1);  // tasks per C tile
-    const int ms = (!scale_only && c.beta != 0.0 && nchain >= 2) ? add_shadow(mc) : -1;
-    Versions V;
-    V.e = &entries_;
+    int ms = (!scale_only && c.beta != 0.0 && nchain >= 2) ? add_shadow(mc) : -1;
     std::vector<Task> tasks;
-    auto opnd = [&](int mat, int64_t r, int64_t l) {  // tile (r, l) of op(X), X n x k
-        return tr ? key_of(mat, l, r) : key_of(mat, r, l);
-    };
-    for (int64_t j = 0; j < tn; ++j) {
-        for (int64_t i = 0; i < tn; ++i) {
-            if (lower ? (i < j) : (i > j)) continue;
-            const bool dg = (i == j);
-            int keyC = key_of(mc, i, j);
-            int64_t mt = std::min(T, n - i * T), nt = std::min(T, n - j * T);
-            if (scale_only) {
-                Task t;
-                t.gpu = owner_tri(i, j, lower, tn);
-                t.op = XK_OP_SCALE;
-                t.tri = dg ? tri : 0;
-                t.out_key = keyC;
-                if (c.beta != 0.0 || dg) t.in.push_back({keyC, V.get(keyC), 2});
-                t.out_ver = V.bump(keyC);
-                t.beta = c.beta;
-                t.tk = -1;
-                t.i = i; t.j = j;
-                t.m = mt; t.n = nt;
-                t.flops = mt * nt;
-                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
-                std::copy(sk, sk + 5, t.skey);
-                tasks.push_back(t);
-                continue;
-            }
-            bool first = true;
-            // diagonal tiles are always read in place (reading R5), off-diagonal ones defer beta
-            const bool defer = ms >= 0 && !dg && defer_beta(keyC);
-            const int keyS = defer ? key_of(ms, i, j) : -1;
-            int64_t pos = 0;
-            for (int64_t l = 0; l < tkn; ++l) {
-                int64_t kt = std::min(T, k - l * T);
-                for (int s = 0; s < (two ? 2 : 1); ++s, ++pos) {
-                    // SYRK: op(A)_i op(A)_j^T.  SYR2K: s=0 op(A)_i op(B)_j^T, s=1 op(B)_i op(A)_j^T
-                    int xa = (two && s == 1) ? mb : ma, xb = (two && s == 0) ? mb : ma;
-                    int keyA = opnd(xa, i, l), keyB = opnd(xb, j, l);
+    for (;;) {  // with the shadow if it fits (fits()), else without
+        Versions V;
+        V.e = &entries_;
+        tasks.clear();
+        auto opnd = [&](int mat, int64_t r, int64_t l) {  // tile (r, l) of op(X), X n x k
+            return tr ? key_of(mat, l, r) : key_of(mat, r, l);
+        };
+        for (int64_t j = 0; j < tn; ++j) {
+            for (int64_t i = 0; i < tn; ++i) {
+                if (lower ? (i < j) : (i > j)) continue;
+                const bool dg = (i == j);
+                int keyC = key_of(mc, i, j);
+                int64_t mt = std::min(T, n - i * T), nt = std::min(T, n - j * T);
+                if (scale_only) {
                     Task t;
                     t.gpu = owner_tri(i, j, lower, tn);
-                    t.op = dg ? XK_OP_GEMM_TRI : XK_OP_GEMM;
+                    t.op = XK_OP_SCALE;
                     t.tri = dg ? tri : 0;
                     t.out_key = keyC;
-                    t.in.push_back({keyA, V.get(keyA), xa == ma ? 0 : 1});
-                    t.in.push_back({keyB, V.get(keyB), xb == ma ? 0 : 1});
-                    if (!first || (c.beta != 0.0 && !defer) || dg) t.in.push_back({keyC, V.get(keyC), 2});
-                    if (defer && pos == nchain - 1) {
-                        t.in.push_back({keyS, V.get(keyS), 2});
-                        t.keyC2 = keyS;
-                        t.beta2 = c.beta;
-                    }
+                    if (c.beta != 0.0 || dg) t.in.push_back({keyC, V.get(keyC), 2});
                     t.out_ver = V.bump(keyC);
-                    t.keyA = keyA;
-                    t.keyB = keyB;
-                    t.ta = tr ? 'T' : 'N';  // op(A) tile = X(i,l) or X(l,i)^T
-                    t.tb = tr ? 'N' : 'T';  // op(B) tile = X(j,l)^T or X(l,j)
-                    t.alpha = c.alpha;
-                    t.beta = first ? (defer ? 0.0 : c.beta) : 1.0;
-                    t.tk = l;
+                    t.beta = c.beta;
+                    t.tk = -1;
                     t.i = i; t.j = j;
-                    t.m = mt; t.n = nt; t.k = kt;
-                    t.flops = dg ? kt * nt * (nt + 1) : 2 * mt * nt * kt;
-                    // staggered chains (reading Q12'), as for DGEMM
-                    int64_t sk[5] = {2 * (l + (i + j) % tkn) + s, (i + j + l) % tmod, i, j, 0};
+                    t.m = mt; t.n = nt;
+                    t.flops = mt * nt;
+                    int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
                     std::copy(sk, sk + 5, t.skey);
                     tasks.push_back(t);
-                    first = false;
+                    continue;
+                }
+                bool first = true;
+                // diagonal tiles are always read in place (reading R5), off-diagonal ones defer beta
+                const bool defer = ms >= 0 && !dg && defer_beta(keyC);
+                const int keyS = defer ? key_of(ms, i, j) : -1;
+                int64_t pos = 0;
+                for (int64_t l = 0; l < tkn; ++l) {
+                    int64_t kt = std::min(T, k - l * T);
+                    for (int s = 0; s < (two ? 2 : 1); ++s, ++pos) {
+                        // SYRK: op(A)_i op(A)_j^T.  SYR2K: s=0 op(A)_i op(B)_j^T, s=1 op(B)_i op(A)_j^T
+                        int xa = (two && s == 1) ? mb : ma, xb = (two && s == 0) ? mb : ma;
+                        int keyA = opnd(xa, i, l), keyB = opnd(xb, j, l);
+                        Task t;
+                        t.gpu = owner_tri(i, j, lower, tn);
+                        t.op = dg ? XK_OP_GEMM_TRI : XK_OP_GEMM;
+                        t.tri = dg ? tri : 0;
+                        t.out_key = keyC;
+                        t.in.push_back({keyA, V.get(keyA), xa == ma ? 0 : 1});
+                        t.in.push_back({keyB, V.get(keyB), xb == ma ? 0 : 1});
+                        if (!first || (c.beta != 0.0 && !defer) || dg) t.in.push_back({keyC, V.get(keyC), 2});
+                        if (defer && pos == nchain - 1) {
+                            t.in.push_back({keyS, V.get(keyS), 2});
+                            t.keyC2 = keyS;
+                            t.beta2 = c.beta;
+                        }
+                        t.out_ver = V.bump(keyC);
+                        t.keyA = keyA;
+                        t.keyB = keyB;
+                        t.ta = tr ? 'T' : 'N';  // op(A) tile = X(i,l) or X(l,i)^T
+                        t.tb = tr ? 'N' : 'T';  // op(B) tile = X(j,l)^T or X(l,j)
+                        t.alpha = c.alpha;
+                        t.beta = first ? (defer ? 0.0 : c.beta) : 1.0;
+                        t.tk = l;
+                        t.i = i; t.j = j;
+                        t.m = mt; t.n = nt; t.k = kt;
+                        t.flops = dg ? kt * nt * (nt + 1) : 2 * mt * nt * kt;
+                        // staggered chains (reading Q12'), as for DGEMM
+                        int64_t sk[5] = {2 * (l + (i + j) % tkn) + s, (i + j + l) % tmod, i, j, 0};
+                        std::copy(sk, sk + 5, t.skey);
+                        tasks.push_back(t);
+                        first = false;
+                    }
                 }
             }
         }
+        if (ms >= 0 && !fits(tasks)) {
+            drop_shadow(ms);
+            ms = -1;
+            continue;
+        }
+        break;
     }
     int rc = run_tasks(tasks, c.sync != 0, out, err);
     drop_shadow(ms);
@@ -706,89 +751,98 @@ int Planner::plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &e
     }
     const int64_t tm = cdiv(m, T), tn = cdiv(n, T), tl = cdiv(ka, T);
     const int64_t tmod = std::max<int64_t>(1, std::max(tm, tn));
-    const int ms = (!scale_only && c.beta != 0.0 && tl >= 2) ? add_shadow(mc) : -1;
-    Versions V;
-    V.e = &entries_;
+    int ms = (!scale_only && c.beta != 0.0 && tl >= 2) ? add_shadow(mc) : -1;
     std::vector<Task> tasks;
-    for (int64_t j = 0; j < tn; ++j) {
-        for (int64_t i = 0; i < tm; ++i) {
-            int keyC = key_of(mc, i, j);
-            int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
-            if (scale_only) {
-                Task t;
-                t.gpu = owner(i, j);
-                t.op = XK_OP_SCALE;
-                t.out_key = keyC;
-                if (c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
-                t.out_ver = V.bump(keyC);
-                t.beta = c.beta;
-                t.tk = -1;
-                t.i = i; t.j = j;
-                t.m = mt; t.n = nt;
-                t.flops = mt * nt;
-                int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
-                std::copy(sk, sk + 5, t.skey);
-                tasks.push_back(t);
-                continue;
-            }
-            // beta deferral when the chain's last task is a GEMM (SYMM_DIAG reads C in place)
-            const bool last_diag = left ? (i == tl - 1) : (j == tl - 1);
-            const bool defer = ms >= 0 && !last_diag && defer_beta(keyC);
-            const int keyS = defer ? key_of(ms, i, j) : -1;
-            for (int64_t l = 0; l < tl; ++l) {
-                int64_t kt = std::min(T, ka - l * T);
-                // sym(A) tile (r, q): stored (r, q) if it lies in the uplo triangle, else (q, r)^T
-                int64_t r = left ? i : l, q = left ? l : j;
-                bool in_tri = lower ? (r >= q) : (r <= q);
-                int keyAt = in_tri ? key_of(ma, r, q) : key_of(ma, q, r);
-                int keyBt = left ? key_of(mb, l, j) : key_of(mb, i, l);
-                Task t;
-                t.gpu = owner(i, j);
-                t.out_key = keyC;
-                t.side = left ? 'L' : 'R';
-                t.uplo = lower ? 'L' : 'U';
-                if (r == q) {
-                    t.op = XK_OP_SYMM_DIAG;
-                    t.keyA = keyAt;
-                    t.keyB = keyBt;
-                    t.in.push_back({keyAt, V.get(keyAt), 0});
-                    t.in.push_back({keyBt, V.get(keyBt), 1});
-                } else if (left) {
-                    t.op = XK_OP_GEMM;
-                    t.keyA = keyAt;
-                    t.keyB = keyBt;
-                    t.ta = in_tri ? 'N' : 'T';
-                    t.tb = 'N';
-                    t.in.push_back({keyAt, V.get(keyAt), 0});
-                    t.in.push_back({keyBt, V.get(keyBt), 1});
-                } else {
-                    t.op = XK_OP_GEMM;  // C(i,j) += B(i,l) * sym(A)(l,j)
-                    t.keyA = keyBt;
-                    t.keyB = keyAt;
-                    t.ta = 'N';
-                    t.tb = in_tri ? 'N' : 'T';
-                    t.in.push_back({keyBt, V.get(keyBt), 1});
-                    t.in.push_back({keyAt, V.get(keyAt), 0});
+    for (;;) {  // with the shadow if it fits (fits()), else without
+        Versions V;
+        V.e = &entries_;
+        tasks.clear();
+        for (int64_t j = 0; j < tn; ++j) {
+            for (int64_t i = 0; i < tm; ++i) {
+                int keyC = key_of(mc, i, j);
+                int64_t mt = std::min(T, m - i * T), nt = std::min(T, n - j * T);
+                if (scale_only) {
+                    Task t;
+                    t.gpu = owner(i, j);
+                    t.op = XK_OP_SCALE;
+                    t.out_key = keyC;
+                    if (c.beta != 0.0) t.in.push_back({keyC, V.get(keyC), 2});
+                    t.out_ver = V.bump(keyC);
+                    t.beta = c.beta;
+                    t.tk = -1;
+                    t.i = i; t.j = j;
+                    t.m = mt; t.n = nt;
+                    t.flops = mt * nt;
+                    int64_t sk[5] = {0, (i + j) % tmod, i, j, 0};
+                    std::copy(sk, sk + 5, t.skey);
+                    tasks.push_back(t);
+                    continue;
                 }
-                if (l > 0 || (c.beta != 0.0 && !defer)) t.in.push_back({keyC, V.get(keyC), 2});
-                if (defer && l == tl - 1) {
-                    t.in.push_back({keyS, V.get(keyS), 2});
-                    t.keyC2 = keyS;
-                    t.beta2 = c.beta;
+                // beta deferral when the chain's last task is a GEMM (SYMM_DIAG reads C in place)
+                const bool last_diag = left ? (i == tl - 1) : (j == tl - 1);
+                const bool defer = ms >= 0 && !last_diag && defer_beta(keyC);
+                const int keyS = defer ? key_of(ms, i, j) : -1;
+                for (int64_t l = 0; l < tl; ++l) {
+                    int64_t kt = std::min(T, ka - l * T);
+                    // sym(A) tile (r, q): stored (r, q) if it lies in the uplo triangle, else (q, r)^T
+                    int64_t r = left ? i : l, q = left ? l : j;
+                    bool in_tri = lower ? (r >= q) : (r <= q);
+                    int keyAt = in_tri ? key_of(ma, r, q) : key_of(ma, q, r);
+                    int keyBt = left ? key_of(mb, l, j) : key_of(mb, i, l);
+                    Task t;
+                    t.gpu = owner(i, j);
+                    t.out_key = keyC;
+                    t.side = left ? 'L' : 'R';
+                    t.uplo = lower ? 'L' : 'U';
+                    if (r == q) {
+                        t.op = XK_OP_SYMM_DIAG;
+                        t.keyA = keyAt;
+                        t.keyB = keyBt;
+                        t.in.push_back({keyAt, V.get(keyAt), 0});
+                        t.in.push_back({keyBt, V.get(keyBt), 1});
+                    } else if (left) {
+                        t.op = XK_OP_GEMM;
+                        t.keyA = keyAt;
+                        t.keyB = keyBt;
+                        t.ta = in_tri ? 'N' : 'T';
+                        t.tb = 'N';
+                        t.in.push_back({keyAt, V.get(keyAt), 0});
+                        t.in.push_back({keyBt, V.get(keyBt), 1});
+                    } else {
+                        t.op = XK_OP_GEMM;  // C(i,j) += B(i,l) * sym(A)(l,j)
+                        t.keyA = keyBt;
+                        t.keyB = keyAt;
+                        t.ta = 'N';
+                        t.tb = in_tri ? 'N' : 'T';
+                        t.in.push_back({keyBt, V.get(keyBt), 1});
+                        t.in.push_back({keyAt, V.get(keyAt), 0});
+                    }
+                    if (l > 0 || (c.beta != 0.0 && !defer)) t.in.push_back({keyC, V.get(keyC), 2});
+                    if (defer && l == tl - 1) {
+                        t.in.push_back({keyS, V.get(keyS), 2});
+                        t.keyC2 = keyS;
+                        t.beta2 = c.beta;
+                    }
+                    t.out_ver = V.bump(keyC);
+                    t.alpha = c.alpha;
+                    t.beta = (l == 0) ? (defer ? 0.0 : c.beta) : 1.0;
+                    t.tk = l;
+                    t.i = i; t.j = j;
+                    t.m = mt; t.n = nt; t.k = kt;
+                    t.flops = 2 * mt * nt * kt;
+                    // staggered chains (reading Q12'), as for DGEMM
+                    int64_t sk[5] = {l + (i + j) % tl, (i + j + l) % tmod, i, j, 0};
+                    std::copy(sk, sk + 5, t.skey);
+                    tasks.push_back(t);
                 }
-                t.out_ver = V.bump(keyC);
-                t.alpha = c.alpha;
-                t.beta = (l == 0) ? (defer ? 0.0 : c.beta) : 1.0;
-                t.tk = l;
-                t.i = i; t.j = j;
-                t.m = mt; t.n = nt; t.k = kt;
-                t.flops = 2 * mt * nt * kt;
-                // staggered chains (reading Q12'), as for DGEMM
-                int64_t sk[5] = {l + (i + j) % tl, (i + j + l) % tmod, i, j, 0};
-                std::copy(sk, sk + 5, t.skey);
-                tasks.push_back(t);
             }
         }
+        if (ms >= 0 && !fits(tasks)) {
+            drop_shadow(ms);
+            ms = -1;
+            continue;
+        }
+        break;
     }
     int rc = run_tasks(tasks, c.sync != 0, out, err);
     drop_shadow(ms);
@@ -865,57 +919,96 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
     bool sh_ok = !solve && tk >= 2;
     for (int64_t j = 0; j < tn && sh_ok; ++j)
         for (int64_t i = 0; i < tm && sh_ok; ++i) sh_ok = defer_beta(key_of(mc, i, j));
-    const int ms = sh_ok ? add_shadow(mc) : -1;
+    int ms = sh_ok ? add_shadow(mc) : -1;
     if (ms >= 0) mats_[ms].host_once = true;
-    const bool sweep_fwd = ms >= 0 ? !fwd : fwd;
-    for (int64_t s = 0; s < nsteps; ++s) {
-        const int64_t kx = sweep_fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
-        const double a_s = solve ? ((s == 0) ? c.alpha : 1.0) : c.alpha;
-        for (int64_t o = 0; o < other; ++o) {
-            const int64_t bi = left ? kx : o, bj = left ? o : kx;
-            int keyD = opA(kx, kx), keyO = key_of(mc, bi, bj);
-            const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
-            // diagonal task on B(kx, o) (left) / B(o, kx) (right)
-            Task t;
-            t.gpu = owner_trxm(bi, bj, left, solve);
-            t.op = solve ? XK_OP_TRSM_DIAG : XK_OP_TRMM_DIAG;
-            t.out_key = keyO;
-            t.keyA = keyD;
-            t.in.push_back({keyD, V.get(keyD), 0});
-            if (ms >= 0) {
-                const int keyS = key_of(ms, bi, bj);
-                t.in.push_back({keyS, V.get(keyS), 2});
-                t.keyC2 = keyS;  // copied into the output tile, then multiplied in place
-            } else {
-                t.in.push_back({keyO, V.get(keyO), 2});
+    for (;;) {  // with the shadow if it fits (fits()), else in place
+        V.cur.clear();
+        tasks.clear();
+        const bool sweep_fwd = ms >= 0 ? !fwd : fwd;
+        for (int64_t s = 0; s < nsteps; ++s) {
+            const int64_t kx = sweep_fwd ? s : nsteps - 1 - s;  // diagonal tile index of this step
+            const double a_s = solve ? ((s == 0) ? c.alpha : 1.0) : c.alpha;
+            for (int64_t o = 0; o < other; ++o) {
+                const int64_t bi = left ? kx : o, bj = left ? o : kx;
+                int keyD = opA(kx, kx), keyO = key_of(mc, bi, bj);
+                const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
+                // diagonal task on B(kx, o) (left) / B(o, kx) (right)
+                Task t;
+                t.gpu = owner_trxm(bi, bj, left, solve);
+                t.op = solve ? XK_OP_TRSM_DIAG : XK_OP_TRMM_DIAG;
+                t.out_key = keyO;
+                t.keyA = keyD;
+                t.in.push_back({keyD, V.get(keyD), 0});
+                if (ms >= 0) {
+                    const int keyS = key_of(ms, bi, bj);
+                    t.in.push_back({keyS, V.get(keyS), 2});
+                    t.keyC2 = keyS;  // copied into the output tile, then multiplied in place
+                } else {
+                    t.in.push_back({keyO, V.get(keyO), 2});
+                }
+                t.out_ver = V.bump(keyO);
+                t.ta = tA;
+                t.side = left ? 'L' : 'R';
+                t.uplo = lower ? 'L' : 'U';
+                t.diag = up(c.diag);
+                t.alpha = a_s;
+                t.tk = s;
+                t.i = bi; t.j = bj;
+                t.m = mt; t.n = nt; t.k = left ? mt : nt;
+                t.flops = left ? mt * mt * nt : mt * nt * nt;
+                int64_t sk[5] = {s, 0, (bi + bj + s) % tmod, bi, bj};
+                std::copy(sk, sk + 5, t.skey);
+                tasks.push_back(t);
+                // TRMM: this tile's remaining contributions (sources still unmodified)
+                if (!solve) {
+                    // contributions nearest the diagonal first (reading R9): the one that reads
+                    // the tile the next step overwrites comes first, so that step's diagonal
+                    // multiply does not wait for this step's whole chain (WAR)
+                    int64_t ph = 1;
+                    for (int64_t dq = 1; dq < tk; ++dq) {
+                        const bool below = left ? elow : !elow;  // contributing q lie below kx
+                        const int64_t q = below ? kx - dq : kx + dq;
+                        if (q < 0 || q >= tk) break;
+                        const int mb = ms >= 0 ? ms : mc;  // B's input tiles (shadow: R15)
+                        int keyA_ = left ? opA(kx, q) : key_of(mb, bi, q);
+                        int keyB_ = left ? key_of(mb, q, bj) : opA(q, kx);
+                        const int64_t kt = std::min(T, ka - q * T);
+                        Task g;
+                        g.gpu = owner_trxm(bi, bj, left, solve);
+                        g.op = XK_OP_GEMM;
+                        g.out_key = keyO;
+                        g.keyA = keyA_;
+                        g.keyB = keyB_;
+                        g.ta = left ? tA : 'N';
+                        g.tb = left ? 'N' : tA;
+                        g.in.push_back({keyA_, V.get(keyA_), left ? 0 : 2});
+                        g.in.push_back({keyB_, V.get(keyB_), left ? 2 : 0});
+                        g.in.push_back({keyO, V.get(keyO), 2});
+                        g.out_ver = V.bump(keyO);
+                        g.alpha = c.alpha;
+                        g.beta = 1.0;
+                        g.tk = s;
+                        g.i = bi; g.j = bj;
+                        g.m = mt; g.n = nt; g.k = kt;
+                        g.flops = 2 * mt * nt * kt;
+                        int64_t sk2[5] = {s, ph++, (bi + bj + s) % tmod, bi, bj};
+                        std::copy(sk2, sk2 + 5, g.skey);
+                        tasks.push_back(g);
+                    }
+                }
             }
-            t.out_ver = V.bump(keyO);
-            t.ta = tA;
-            t.side = left ? 'L' : 'R';
-            t.uplo = lower ? 'L' : 'U';
-            t.diag = up(c.diag);
-            t.alpha = a_s;
-            t.tk = s;
-            t.i = bi; t.j = bj;
-            t.m = mt; t.n = nt; t.k = left ? mt : nt;
-            t.flops = left ? mt * mt * nt : mt * nt * nt;
-            int64_t sk[5] = {s, 0, (bi + bj + s) % tmod, bi, bj};
-            std::copy(sk, sk + 5, t.skey);
-            tasks.push_back(t);
-            // TRMM: this tile's remaining contributions (sources still unmodified)
-            if (!solve) {
-                // contributions nearest the diagonal first (reading R9): the one that reads
-                // the tile the next step overwrites comes first, so that step's diagonal
-                // multiply does not wait for this step's whole chain (WAR)
-                int64_t ph = 1;
-                for (int64_t dq = 1; dq < tk; ++dq) {
-                    const bool below = left ? elow : !elow;  // contributing q lie below kx
-                    const int64_t q = below ? kx - dq : kx + dq;
-                    if (q < 0 || q >= tk) break;
-                    const int mb = ms >= 0 ? ms : mc;  // B's input tiles (shadow: R15)
-                    int keyA_ = left ? opA(kx, q) : key_of(mb, bi, q);
-                    int keyB_ = left ? key_of(mb, q, bj) : opA(q, kx);
-                    const int64_t kt = std::min(T, ka - q * T);
+            if (!solve) continue;
+            // TRSM: update the rows (cols) still to be solved with the solved tiles of step s
+            for (int64_t r = 0; r < tk; ++r) {
+                const bool later = fwd ? r > kx : r < kx;
+                if (!later) continue;
+                for (int64_t o = 0; o < other; ++o) {
+                    const int64_t bi = left ? r : o, bj = left ? o : r;
+                    int keyO = key_of(mc, bi, bj);
+                    int keyA_ = left ? opA(r, kx) : key_of(mc, bi, kx);
+                    int keyB_ = left ? key_of(mc, kx, bj) : opA(kx, r);
+                    const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
+                    const int64_t kt = std::min(T, ka - kx * T);
                     Task g;
                     g.gpu = owner_trxm(bi, bj, left, solve);
                     g.op = XK_OP_GEMM;
@@ -928,62 +1021,33 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
                     g.in.push_back({keyB_, V.get(keyB_), left ? 2 : 0});
                     g.in.push_back({keyO, V.get(keyO), 2});
                     g.out_ver = V.bump(keyO);
-                    g.alpha = c.alpha;
-                    g.beta = 1.0;
+                    g.alpha = -1.0;
+                    g.beta = a_s;
                     g.tk = s;
                     g.i = bi; g.j = bj;
                     g.m = mt; g.n = nt; g.k = kt;
                     g.flops = 2 * mt * nt * kt;
-                    int64_t sk2[5] = {s, ph++, (bi + bj + s) % tmod, bi, bj};
-                    std::copy(sk2, sk2 + 5, g.skey);
+                    // lookahead (reading R9): the row (col) the next step solves is updated first,
+                    // so its diagonal solve can run while the other updates of this step proceed.
+                    // Update window (reading R10): the row solved at step sr is updated by step s
+                    // at time u = max(s, sr - D), D = 2 x the grid extent along the solved
+                    // dimension; within a time, rows nearest the front first, then s ascending
+                    // (every tile's chain keeps its order: results are those of right-looking)
+                    const int64_t sr = fwd ? r : nsteps - 1 - r;
+                    const int64_t u = std::max<int64_t>(s, sr - Dw);
+                    const int64_t ph = (sr == s + 1) ? 1 : 2;
+                    int64_t sk[5] = {u, ph, sr * nsteps + s, (bi + bj + s) % tmod, o};
+                    std::copy(sk, sk + 5, g.skey);
                     tasks.push_back(g);
                 }
             }
         }
-        if (!solve) continue;
-        // TRSM: update the rows (cols) still to be solved with the solved tiles of step s
-        for (int64_t r = 0; r < tk; ++r) {
-            const bool later = fwd ? r > kx : r < kx;
-            if (!later) continue;
-            for (int64_t o = 0; o < other; ++o) {
-                const int64_t bi = left ? r : o, bj = left ? o : r;
-                int keyO = key_of(mc, bi, bj);
-                int keyA_ = left ? opA(r, kx) : key_of(mc, bi, kx);
-                int keyB_ = left ? key_of(mc, kx, bj) : opA(kx, r);
-                const int64_t mt = std::min(T, m - bi * T), nt = std::min(T, n - bj * T);
-                const int64_t kt = std::min(T, ka - kx * T);
-                Task g;
-                g.gpu = owner_trxm(bi, bj, left, solve);
-                g.op = XK_OP_GEMM;
-                g.out_key = keyO;
-                g.keyA = keyA_;
-                g.keyB = keyB_;
-                g.ta = left ? tA : 'N';
-                g.tb = left ? 'N' : tA;
-                g.in.push_back({keyA_, V.get(keyA_), left ? 0 : 2});
-                g.in.push_back({keyB_, V.get(keyB_), left ? 2 : 0});
-                g.in.push_back({keyO, V.get(keyO), 2});
-                g.out_ver = V.bump(keyO);
-                g.alpha = -1.0;
-                g.beta = a_s;
-                g.tk = s;
-                g.i = bi; g.j = bj;
-                g.m = mt; g.n = nt; g.k = kt;
-                g.flops = 2 * mt * nt * kt;
-                // lookahead (reading R9): the row (col) the next step solves is updated first,
-                // so its diagonal solve can run while the other updates of this step proceed.
-                // Update window (reading R10): the row solved at step sr is updated by step s
-                // at time u = max(s, sr - D), D = 2 x the grid extent along the solved
-                // dimension; within a time, rows nearest the front first, then s ascending
-                // (every tile's chain keeps its order: results are those of right-looking)
-                const int64_t sr = fwd ? r : nsteps - 1 - r;
-                const int64_t u = std::max<int64_t>(s, sr - Dw);
-                const int64_t ph = (sr == s + 1) ? 1 : 2;
-                int64_t sk[5] = {u, ph, sr * nsteps + s, (bi + bj + s) % tmod, o};
-                std::copy(sk, sk + 5, g.skey);
-                tasks.push_back(g);
-            }
+        if (ms >= 0 && !fits(tasks)) {
+            drop_shadow(ms);
+            ms = -1;
+            continue;
         }
+        break;
     }
     int rc = run_tasks(tasks, c.sync != 0, out, err);
     drop_shadow(ms);

@@ -33,6 +33,7 @@ struct Flags {
     int window = 2;
     int P = 1, Q = 1;
     int64_t T = 2048;
+    int64_t mem_bytes = 0;  // tile-cache capacity per GPU the plan must fit (0 = unlimited)
 };
 
 // A host matrix as the planner sees it: identity (base, ld) and stored extent.
@@ -190,6 +191,9 @@ private:
     int add_shadow(int mc);
     bool defer_beta(int keyC) const;
     void drop_shadow(int ms);
+    // capacity check for a shadow plan: every GPU's tiles (resident now + read or written by
+    // this call's tasks on it) fit in flags_.mem_bytes
+    bool fits(const std::vector<Task> &tasks) const;
     int plan_gemm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
     int plan_syrk(const xk_call_t &c, bool two, std::vector<Rec> &out, std::string &err);
     int plan_symm(const xk_call_t &c, std::vector<Rec> &out, std::string &err);

@@ -63,7 +63,7 @@ class Tile:
 
 class Model:
     def __init__(self, bw, rate_mflops=35000000, topo="ranked", optimistic=True, window=2,
-                 grid=(0, 0), tile=2048):
+                 grid=(0, 0), tile=2048, mem_bytes=0):
         self.bw = [list(r) for r in bw]
         self.G = len(bw) - 1
         self.once = set()  # read-once shadow bases (R15)
@@ -74,6 +74,8 @@ class Model:
         self.W = max(1, window)
         self.P, self.Q = grid if grid[0] > 0 else near_square(self.G)
         self.T = tile
+        self.mem = mem_bytes      # per-GPU tile-cache capacity (0 = unlimited)
+        self._no_shadow = False
         self.tiles = {}          # (base, ld, bi, bj) -> Tile
         self.extent = {}         # (base, ld) -> [rows, cols]
         self.link = {}           # (src_idx, dst_idx) -> free time
@@ -172,14 +174,22 @@ class Model:
         ta, tb = transA.upper() in "TC", transB.upper() in "TC"
         lower, left = uplo.upper() == "L", side.upper() == "L"
         if routine in (DGEMM, DSYRK, DSYR2K, DSYMM, DTRMM, DTRSM):
-            if routine == DGEMM:
-                tasks = self.gen_gemm(ta, tb, m, n, k, alpha, beta, A, lda, B, ldb, C, ldc)
-            elif routine in (DSYRK, DSYR2K):
-                tasks = self.gen_syrk(routine == DSYR2K, lower, ta, n, k, alpha, beta, A, lda, B, ldb, C, ldc)
-            elif routine == DSYMM:
-                tasks = self.gen_symm(left, lower, m, n, alpha, beta, A, lda, B, ldb, C, ldc)
-            else:
-                tasks = self.gen_trxm(routine == DTRSM, left, lower, ta, diag.upper(), m, n, alpha, A, lda, C, ldc)
+            def gen():
+                if routine == DGEMM:
+                    return self.gen_gemm(ta, tb, m, n, k, alpha, beta, A, lda, B, ldb, C, ldc)
+                if routine in (DSYRK, DSYR2K):
+                    return self.gen_syrk(routine == DSYR2K, lower, ta, n, k, alpha, beta, A, lda, B, ldb, C, ldc)
+                if routine == DSYMM:
+                    return self.gen_symm(left, lower, m, n, alpha, beta, A, lda, B, ldb, C, ldc)
+                return self.gen_trxm(routine == DTRSM, left, lower, ta, diag.upper(), m, n, alpha, A, lda, C, ldc)
+            self._shadow = None
+            tasks = gen()
+            if tasks and self._shadow is not None and not self.fits(tasks):
+                # the shadow does not fit next to the call's tiles: plan without it
+                self.drop_shadow(ldc)
+                self._no_shadow = True
+                tasks = gen()
+                self._no_shadow = False
             if tasks:
                 self.run(tasks, sync, out)
             if routine in (DGEMM, DSYRK, DSYR2K, DSYMM, DTRMM):
@@ -283,7 +293,24 @@ class Model:
         self._shadow = shadow
         return tasks
 
+    def fits(self, tasks):
+        """Capacity rule of a shadow plan: on every GPU, the tiles resident now plus the
+        tiles its tasks read or write, at 8 * round_up(rows, 16) * cols bytes each, fit."""
+        if self.mem <= 0:
+            return True
+        sets = [dict() for _ in range(self.G)]
+        for t in self.tiles.values():
+            for g in t.gpus:
+                sets[g][id(t)] = t
+        for t in tasks:
+            for tl in [t["out"]] + [x[0] for x in t["ins"]]:
+                sets[t["gpu"]][id(tl)] = tl
+        return all(sum(8 * ceil_div(tl.rows, 16) * 16 * tl.cols for tl in s.values()) <= self.mem
+                   for s in sets)
+
     def new_shadow(self, C, ldc):
+        if self._no_shadow:
+            return None
         self.calls += 1
         shadow = ("shadow", self.calls, C)
         self.extent[(shadow, ldc)] = list(self.extent[(C, ldc)])
@@ -432,7 +459,8 @@ class Model:
         if (not solve and tk >= 2
                 and all(self.host_only(self.tile(C, ldc, i, j)) for j in range(tn) for i in range(tm))):
             shadow = self.new_shadow(C, ldc)
-            self.once.add(shadow)  # read from the host at most once per tile
+            if shadow is not None:
+                self.once.add(shadow)  # read from the host at most once per tile
         Bin = shadow if shadow is not None else C
         sweep_fwd = (not fwd) if shadow is not None else fwd
         for s in range(tk):

@@ -623,3 +623,54 @@ def test_sync_call_keeps_gpu_dirty_inputs(G, second):
              dict(routine=pm.COHERENT, m=N, n=N, C=D_ADDR, ldc=N)]
     got, exp = both(uniform(G), dict(topo="ranked", optimistic=True, window=2, tile=T), calls)
     assert got == exp
+
+
+def _uses_shadow(routine, recs):
+    if routine == "dtrmm":  # shadow sweep is top-down: row 0 multiplied first (R15)
+        return next(r for r in recs if r[1] == pm.TASK and r[15] == pm.OP_TRMM_DIAG)[3] == 0
+    # beta deferred: some chain's first task (tk = 0) does not read C (deps[2] == -1)
+    return any(r[1] == pm.TASK and r[5] == 0 and r[15] == pm.OP_GEMM and r[14][2] == -1 for r in recs)
+
+
+# per-GPU tiles of the shadow plan at G = 1, t = 4, written from the rule (DESIGN Q12'', R15):
+# DGEMM A 16 + B 16 + C 16 + shadow 16; SYR2K (lower) A 16 + B 16 + C triangle 10 + shadow of
+# the 6 off-diagonal tiles; SYMM (left, lower) A triangle 10 + B 16 + C 16 + shadow of the 12
+# tiles whose chain ends in a GEMM (rows 0..2); TRMM A triangle 10 + B 16 + shadow 16
+SHADOW_TILES_G1 = {"dgemm": 64, "dsyr2k": 48, "dsymm": 54, "dtrmm": 42}
+
+
+@pytest.mark.parametrize("routine", ["dgemm", "dsyr2k", "dsymm", "dtrmm"])
+@pytest.mark.parametrize("G", [1, 4])
+def test_shadow_only_when_it_fits(routine, G):
+    """a per-call shadow (beta deferral Q12'', TRMM R15) adds a second copy
+    of C (B) to the device footprint.  With a capacity below footprint + shadow the call is
+    planned without it; with room it keeps it.  G = 1: the threshold is the closed form above
+    (tiles of T = 4 take 8*16*4 = 512 bytes).  G = 4: the planner's own threshold, where the
+    model must agree record for record on both sides of it."""
+    T, t = 4, 4
+    N = T * t
+    tile = 8 * 16 * T
+    call = {"dgemm": gemm(m=N, n=N, k=N, lda=N, ldb=N, ldc=N),
+            "dsyr2k": dict(routine=pm.DSYR2K, uplo="L", transA="N", n=N, k=N, alpha=1.5, beta=-0.75,
+                           A=A_ADDR, lda=N, B=B_ADDR, ldb=N, C=C_ADDR, ldc=N, sync=True),
+            "dsymm": dict(routine=pm.DSYMM, side="L", uplo="L", m=N, n=N, alpha=1.5, beta=-0.75,
+                          A=A_ADDR, lda=N, B=B_ADDR, ldb=N, C=C_ADDR, ldc=N, sync=True),
+            "dtrmm": dict(routine=pm.DTRMM, side="L", uplo="L", transA="N", diag="N", m=N, n=N,
+                          alpha=1.5, A=A_ADDR, lda=N, C=C_ADDR, ldc=N, sync=True)}[routine]
+
+    def plan(mem):
+        return xk.plan_dump(xk.make_call(**call), uniform(G), tile=T, mem_bytes=mem)
+    if G == 1:
+        need = SHADOW_TILES_G1[routine] * tile
+    else:
+        lo, hi = 1, 1 << 30  # smallest capacity that keeps the shadow
+        while lo < hi:
+            mid = (lo + hi) // 2
+            lo, hi = (lo, mid) if _uses_shadow(routine, plan(mid)) else (mid + 1, hi)
+        need = lo
+    assert _uses_shadow(routine, plan(0))  # unlimited
+    for mem, expect in ((need, True), (need - 1, False)):
+        got, exp = both(uniform(G), dict(topo="ranked", optimistic=True, window=2, tile=T,
+                                         mem_bytes=mem), [call])
+        assert got == exp
+        assert _uses_shadow(routine, got[0]) == expect, (mem, need)
