@@ -9,14 +9,20 @@ splitmix64 generator (uniform [-1,1)), owner grid near-square 
 
 A step is one whole DGEMM (every §8(a) row: tiling, owner map, directory, source
 selection, transfers, tile kernels, coherence):
-  value : data-on-device -- A, B, C already resident in HBM (prefetched into the tile
-          cache, untimed); one xk_dgemm_async + xk_sync per step, C updated on the GPUs.
-  e2e   : the paper's host-resident measurement -- xk_dgemm (synchronous) from pinned
-          host buffers; every step copies A, B, C tiles H2D and C D2H inside the timed
-          region and ends with C coherent on the host.
-Timing: CUDA events on a side stream with a full device synchronize on both sides of the
-K timed steps (the library's work spans its own H2D/D2H/P2P/kernel streams), barrier and
-max over ranks under torchrun.  Inputs (8.6 GB per matrix) are far larger than L2 (126 MB).
+  value : the metric, end to end -- xk_dgemm (synchronous) from pinned host buffers; every
+          step copies A, B, C tiles H2D and C D2H inside the timed region and ends with C
+          coherent on the host.  CUDA events + a full device
+          synchronize on both sides of the K steps, barrier and max over ranks.
+  e2e   : the same K calls timed by the host wall clock (API entry to return), with the
+          H2D/D2H bytes per step and the fraction of the e2e roofline, the
+          host-link terms taken from a concurrent probe of all GPUs' links.
+  data_on_device : A, B, C already resident in HBM (prefetched, untimed); xk_dgemm_async +
+          xk_sync per step (paper §IV-C, Table II "data on device").
+  roofline : the tile kernel (grouped launch) timed by CUDA events in a second pass of the
+          data-on-device steps, against the FP64 peak.
+  ablation (G > 1) : BASELINE configs[1], N=16384 T=2048, every heuristic mode (paper Table II).
+  north_star (G = 8, or --north-star) : N=65536 T=4096 host-resident vs 70% of G x FP64 peak.
+Inputs (8.6 GB per matrix) are far larger than L2 (126 MB): no flush needed.
 
 Multi-GPU: under torchrun the library runs in rank mode -- one process per GPU.  The host
 matrices live in /dev/shm file mappings shared by the processes; every xk call is
@@ -59,7 +65,12 @@ def parse():
     ap.add_argument("--optimistic", type=int, default=1)
     ap.add_argument("--kstreams", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-ablation", action="store_true", help="skip the N>1 heuristic ablation")
+    ap.add_argument("--north-star", action="store_true", help="run the N=65536 north-star point at any G")
+    ap.add_argument("--no-north-star", action="store_true")
+    ap.add_argument("--ns-n", type=int, default=65536, help="north-star N (default 65536)")
+    ap.add_argument("--host-probe-mib", type=int, default=4096,
+                    help="bytes per GPU per direction of the concurrent host-link probe")
     return ap.parse_args()
 
 
@@ -272,14 +283,14 @@ def share_inputs(N, rank, ws):
     per GPU): file mappings every process maps (the library's "host memory" is shared by its
     processes) -- files in /dev/shm when it has room, else anonymous memfds that the other
     ranks open through /proc/<rank 0>/fd (a small /dev/shm mount must not cap the run);
-    rank 0 fills them, the others map them after a barrier.  Returns (A, B, C, paths) with
-    the session-file path last; only real files in the list are unlinked at the end."""
+    rank 0 fills them, the others map them after a barrier.  Returns (A, B, C, paths, base):
+    only real files in `paths` are unlinked at the end; `base` names the session files."""
     import inputs
+    import paper_conf_sc_gautierl21_b200 as xk
     if ws == 1:
         A, B, C = make_inputs(N)
-        return A, B, C, []
+        return A, B, C, [], None
     import torch.distributed as dist
-    import paper_conf_sc_gautierl21_b200 as xk
     obj = [None]
     if rank == 0:
         base = xk.new_session_path("xkbench")
@@ -294,20 +305,20 @@ def share_inputs(N, rank, ws):
             for p in paths:
                 xk.shared_matrix(p, N, N, create=True)
         else:
-            global _MEMFDS
-            _MEMFDS = [os.memfd_create("xkbench" + s) for s in "ABC"]
-            for fd in _MEMFDS:
+            fds = [os.memfd_create("xkbench%d%s" % (N, s)) for s in "ABC"]
+            _MEMFDS.extend(fds)
+            for fd in fds:
                 os.ftruncate(fd, N * N * 8)
-            paths = ["/proc/%d/fd/%d" % (os.getpid(), fd) for fd in _MEMFDS]
-        obj = [paths + [base + ".session"]]
+            paths = ["/proc/%d/fd/%d" % (os.getpid(), fd) for fd in fds]
+        obj = [(paths, base)]
     dist.broadcast_object_list(obj, src=0, group=_HOST_GROUP)
-    paths = obj[0]
-    mats = [xk.shared_matrix(p, N, N, create=False) for p in paths[:3]]
+    paths, base = obj[0]
+    mats = [xk.shared_matrix(p, N, N, create=False) for p in paths]
     if rank == 0:
         for M, seed in zip(mats, (inputs.SEED_A, inputs.SEED_B, inputs.SEED_C)):
             inputs.uniform(seed, N, N, out=M)
     barrier(ws)
-    return mats[0], mats[1], mats[2], [p for p in paths if not p.startswith("/proc/")]
+    return mats[0], mats[1], mats[2], [p for p in paths if not p.startswith("/proc/")], base
 
 
 _MEMFDS = []
@@ -323,28 +334,178 @@ def sum_over_ranks(vals, ws):
     return t.tolist()
 
 
+def gather_per_gpu(v, ws):
+    """Rank mode: every rank's own value, in rank order (rank r drives GPU r)."""
+    if ws == 1:
+        return [v]
+    vec = [0.0] * ws
+    vec[int(os.environ.get("RANK", "0"))] = float(v)
+    return sum_over_ranks(vec, ws)
+
+
+class Lib:
+    """One library session (xk_init .. xk_finalize) of the run; rank mode gets a fresh
+    session file per (re-)initialisation (the heuristic ablation re-initialises per mode)."""
+
+    def __init__(self, args, rank, ws, base):
+        self.args, self.rank, self.ws, self.base, self.n = args, rank, ws, base, 0
+
+    def init(self, mats, tile, topo="ranked", optimistic=True, probe=True):
+        import paper_conf_sc_gautierl21_b200 as xk
+        kw = dict(tile=tile, topo=topo, optimistic=bool(optimistic), kstreams=self.args.kstreams, probe=probe)
+        if self.ws > 1:
+            self.n += 1
+            xk.init(rank=self.rank, world=self.ws, session="%s.session%d" % (self.base, self.n), **kw)
+        else:
+            xk.init(ngpus=self.args.gpus, **kw)
+        for X in mats:
+            xk.register(X)
+        return xk
+
+
+def host_step_bytes(xk, steps, ws):
+    se = xk.get_stats()
+    mine = [sum(se["h2d_bytes"]), sum(se["d2h_bytes"]), sum(se["p2p_in_bytes"])]
+    per_gpu_h2d = se["h2d_bytes"][:se["ngpus"]] if ws == 1 else gather_per_gpu(se["h2d_bytes"][int(os.environ.get("RANK", "0"))], ws)
+    tot = [int(v) // steps for v in sum_over_ranks(mine, ws)]
+    return tot[0], tot[1], tot[2], [int(v) // steps for v in per_gpu_h2d]
+
+
+def timed_host_resident(xk, A, B, C, N, T, steps, warmup, ws, timer, clocks=None, rank=0, gpus=1):
+    """xk_dgemm from pinned host memory: every H2D/D2H inside the timed region, C coherent on
+    the host at the end of each call.  Device time (CUDA events, full device synchronize on
+    both sides, max over ranks) and host wall time of the API calls."""
+    flops = 2.0 * N * N * N
+    for _ in range(warmup):
+        xk.dgemm("N", "N", N, N, N, ALPHA, A, A.strides[1] // 8, B, B.strides[1] // 8, BETA, C, C.strides[1] // 8)
+    xk.reset_stats()
+    barrier(ws)
+    if clocks is not None and rank == 0:
+        clocks.start()
+    wall = 0.0
+    timer.start()
+    for _ in range(steps):
+        t0 = time.perf_counter()
+        xk.dgemm("N", "N", N, N, N, ALPHA, A, A.strides[1] // 8, B, B.strides[1] // 8, BETA, C, C.strides[1] // 8)
+        wall += time.perf_counter() - t0
+    ms = max_over_ranks(timer.stop_ms(), ws)
+    wall_ms = max_over_ranks(1000.0 * wall, ws)
+    barrier(ws)
+    clk = clocks.stop(gpus) if (clocks is not None and rank == 0) else None
+    launches = int(sum_over_ranks([xk.get_stats()["kernel_launches"]], ws)[0])
+    h2d, d2h, p2p, per_gpu = host_step_bytes(xk, steps, ws)
+    return {"tflops": steps * flops / (ms * 1e-3) / 1e12, "ms": ms / steps,
+            "wall_tflops": steps * flops / (wall_ms * 1e-3) / 1e12, "wall_ms": wall_ms / steps,
+            "h2d": h2d, "d2h": d2h, "p2p": p2p, "h2d_per_gpu": per_gpu, "launches": launches, "clocks": clk}
+
+
+def e2e_roofline(topo, G, N, h2d, d2h, p2p):
+    """T_roof = max(F/(G*P64), B_h2d/BW_h2d(G), B_d2h/BW_d2h(G), (B_h2d+B_d2h)/BW_duplex(G),
+    B_p2p/BW_p2p(G)); BW_*(G) = all GPUs copying at once (probed by
+    xk_probe_host_links), BW_p2p(G) = G x the slowest probed peer link."""
+    flops = 2.0 * N * N * N
+    ha = topo.get("host_all_MBps") or {}
+    if ha.get("h2d"):
+        bw_h2d, bw_d2h, bw_dup = ha["h2d"] * 1e6, ha["d2h"] * 1e6, ha["duplex"] * 1e6
+        src = "concurrent probe (all %d GPU(s) at once, %d MiB per GPU per direction)" % (
+            G, topo.get("host_probe_bytes", 0) >> 20)
+    else:
+        bw_h2d = min(topo["bw_MBps"][G][g] for g in range(G)) * 1e6 * G
+        bw_d2h = min(topo["bw_MBps"][g][G] for g in range(G)) * 1e6 * G
+        bw_dup = bw_h2d + bw_d2h
+        src = "G x the per-GPU probe (no concurrent probe)"
+    terms = {"fp64": flops / (G * FP64_PEAK_TFLOPS * 1e12), "h2d": h2d / bw_h2d, "d2h": d2h / bw_d2h,
+             "duplex": (h2d + d2h) / bw_dup}
+    if G > 1 and p2p:
+        peer = min(topo["bw_MBps"][s][d] for s in range(G) for d in range(G) if s != d) * 1e6
+        terms["p2p"] = p2p / (peer * G)
+    return max(terms.values()), {k: round(v * 1e3, 3) for k, v in terms.items()}, src
+
+
+ABLATION_MODES = (("full", "ranked", True), ("no_optimistic", "ranked", False),
+                  ("no_optimistic_no_topo", "unranked", False), ("home", "home", True))
+
+
+def run_ablation(lib, A, B, C, ws, timer, N=16384, T=2048, steps=2):
+    """Paper Table II / BASELINE configs[1]: DGEMM N=16384, T=2048 host-resident, every
+    heuristic mode (one library session each), 1 warm-up + `steps` timed calls; TF/s and
+    H2D bytes per GPU.  The N x N operands are views of the bench matrices (ld = their N)."""
+    out = {"config": "DGEMM N=%d tile %d NN alpha=1.5 beta=-0.75 host-resident, %d GPU(s)" % (N, T, lib.args.gpus if ws == 1 else ws)}
+    Av, Bv, Cv = A[:N, :N], B[:N, :N], C[:N, :N]
+    for name, topo, opt in ABLATION_MODES:
+        xk = lib.init((A, B, C), T, topo=topo, optimistic=opt)
+        r = timed_host_resident(xk, Av, Bv, Cv, N, T, steps, 1, ws, timer)
+        xk.finalize()
+        out[name] = {"tflops": r["tflops"], "ms_per_step": r["ms"], "h2d_bytes": r["h2d"],
+                     "p2p_bytes": r["p2p"], "h2d_bytes_per_gpu": r["h2d_per_gpu"]}
+    full = out["full"]["tflops"]
+    for name, _, _ in ABLATION_MODES[1:]:
+        out[name]["vs_full"] = out[name]["tflops"] / full - 1.0
+    return out
+
+
+def host_mem_available():
+    try:
+        with open("/proc/meminfo") as f:
+            for ln in f:
+                if ln.startswith("MemAvailable:"):
+                    return int(ln.split()[1]) * 1024
+    except OSError:
+        pass
+    return 0
+
+
+def run_north_star(args, rank, ws, timer, N=65536, T=4096, steps=2):
+    """north_star: host-resident DGEMM N=65536, T=4096 on all GPUs, 1 warm-up + 2 steps;
+    fraction of G x the FP64 peak (target >= 0.70)."""
+    G = ws if ws > 1 else args.gpus
+    need = 3 * N * N * 8
+    ok = host_mem_available() > 1.15 * need
+    ok = sum_over_ranks([1.0 if ok else 0.0], ws)[0] == ws
+    if not ok:
+        return {"skipped": "host memory: %d GB needed for A, B, C" % (need >> 30)}
+    A, B, C, paths, base = share_inputs(N, rank, ws)
+    try:
+        lib = Lib(args, rank, ws, base or "")
+        xk = lib.init((A, B, C), T)
+        xk.probe_host_links(1 << 30)
+        topo = xk.get_topology()
+        r = timed_host_resident(xk, A, B, C, N, T, steps, 1, ws, timer)
+        xk.finalize()
+    finally:
+        barrier(ws)
+        if rank == 0:
+            for p in paths:
+                if os.path.exists(p):
+                    os.unlink(p)
+    t_roof, terms, src = e2e_roofline(topo, G, N, r["h2d"], r["d2h"], r["p2p"])
+    return {"config": "DGEMM N=%d tile %d NN host-resident on %d GPU(s)" % (N, T, G), "tflops": r["tflops"],
+            "ms_per_step": r["ms"], "frac_of_fp64_peak": r["tflops"] / (G * FP64_PEAK_TFLOPS),
+            "target_frac": 0.70, "roofline_frac": t_roof / (r["ms"] * 1e-3), "roofline_terms_ms": terms,
+            "h2d_bytes_per_step": r["h2d"], "d2h_bytes_per_step": r["d2h"], "p2p_bytes_per_step": r["p2p"]}
+
+
 def run_xk(args, rank, ws):
     """ws == 1: one process drives the GPU(s) (--gpus G > 1 = the single-process multi-GPU
     runtime).  Under torchrun (ws > 1): rank mode -- one process per GPU, every xk call
     collective, each process executing its own GPU's part of the identical plan."""
-    import torch
-    import paper_conf_sc_gautierl21_b200 as xk
     G = ws if ws > 1 else args.gpus
     N, T = args.n, args.tile
     flops = 2.0 * N * N * N
-    A, B, C, paths = share_inputs(N, rank, ws)
-    kw = dict(tile=T, topo=args.topo, optimistic=bool(args.optimistic), kstreams=args.kstreams, probe=True)
-    if ws > 1:
-        xk.init(rank=rank, world=ws, session=paths[-1], **kw)
-    else:
-        xk.init(ngpus=G, **kw)
-    for X in (A, B, C):
-        xk.register(X)
+    A, B, C, paths, base = share_inputs(N, rank, ws)
+    lib = Lib(args, rank, ws, base)
+    xk = lib.init((A, B, C), T)
+    # SURVEY §8(d): host links with every GPU copying at once (untimed set-up, like a1)
+    xk.probe_host_links(args.host_probe_mib << 20)
     topo = xk.get_topology()
     timer = DevTimer()
     clocks = ClockSampler()
 
-    # ---------------- value: data-on-device (A, B, C resident in HBM)
+    # ---------------- value: the metric, host-resident end to end through xk_dgemm
+    host = timed_host_resident(xk, A, B, C, N, T, args.steps, args.warmup, ws, timer, clocks, rank, G)
+    t_roof, terms, bw_src = e2e_roofline(topo, G, N, host["h2d"], host["d2h"], host["p2p"])
+
+    # ---------------- data-on-device: A, B, C resident in HBM (prefetched, untimed)
     for X in (A, B, C):
         xk.memory_prefetch_async(N, N, X, N)
     xk.sync()
@@ -353,16 +514,13 @@ def run_xk(args, rank, ws):
         xk.sync()
     xk.reset_stats()
     barrier(ws)
-    if rank == 0:
-        clocks.start()
     timer.start()
     for _ in range(args.steps):
         xk.dgemm_async("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
         xk.sync()
-    ms = max_over_ranks(timer.stop_ms(), ws)
+    ms_dod = max_over_ranks(timer.stop_ms(), ws)
     barrier(ws)
-    clk = clocks.stop(G) if rank == 0 else None
-    launches = int(sum_over_ranks([xk.get_stats()["kernel_launches"]], ws)[0])
+    dod_launches = int(sum_over_ranks([xk.get_stats()["kernel_launches"]], ws)[0])
     # roofline pass: the same K steps with every grouped launch timed by CUDA events on its
     # kernel stream (timing serialises launches, so each duration is the kernel's own)
     xk.reset_stats()
@@ -377,37 +535,37 @@ def run_xk(args, rank, ws):
     xk.memory_coherent_sync(N, N, C, N)
     for X in (C, A, B):
         xk.memory_invalidate(N, N, X, N)
-    value = args.steps * flops / (ms * 1e-3) / 1e12
+    xk.finalize()
+    dod = {"value": args.steps * flops / (ms_dod * 1e-3) / 1e12, "unit": "TFLOP/s",
+           "ms_per_step": ms_dod / args.steps, "gpu_launches": dod_launches,
+           "mode": "A, B, C resident in HBM (prefetched, untimed); xk_dgemm_async + xk_sync per step, "
+                   "C updated on the GPUs (no host traffic)"}
 
-    # ---------------- e2e: host-resident, H2D + D2H inside the timed region
-    e2e = None
-    if not args.no_e2e:
-        for _ in range(max(1, args.warmup - 1)):
-            xk.dgemm("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-        xk.reset_stats()
-        barrier(ws)
-        timer.start()
-        for _ in range(args.steps):
-            xk.dgemm("N", "N", N, N, N, ALPHA, A, N, B, N, BETA, C, N)
-        ms_e2e = max_over_ranks(timer.stop_ms(), ws)
-        se = xk.get_stats()
-        mine = [sum(se["h2d_bytes"]), sum(se["d2h_bytes"]), sum(se["p2p_in_bytes"])]
-        h2d, d2h, p2p = (int(v) // args.steps for v in sum_over_ranks(mine, ws))
-        tf_e2e = args.steps * flops / (ms_e2e * 1e-3) / 1e12
-        bw_h2d = min(topo["bw_MBps"][G][g] for g in range(G)) * 1e6 * G
-        bw_d2h = min(topo["bw_MBps"][g][G] for g in range(G)) * 1e6 * G
-        t_roof = max(flops / (G * FP64_PEAK_TFLOPS * 1e12), h2d / bw_h2d, d2h / bw_d2h)
-        e2e = {"value": tf_e2e, "unit": "TFLOP/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-               "ms_per_step": ms_e2e / args.steps, "p2p_bytes_per_step": p2p,
-               "roofline_frac": t_roof / (ms_e2e * 1e-3 / args.steps),
-               "roofline": "max(F/(G*P64), B_h2d/BW_h2d, B_d2h/BW_d2h) with P64=%.1f TFLOP/s/GPU and the "
-                           "probed PCIe bandwidths" % FP64_PEAK_TFLOPS}
+    ablation = run_ablation(lib, A, B, C, ws, timer) if (G > 1 and not args.no_ablation and N >= 16384) else None
+    cpu = cpu_baseline(N, A, B, C) if (rank == 0 and not args.no_cpu_baseline and ws == 1) else None
+    barrier(ws)
+    if rank == 0:
+        for p in paths:
+            if os.path.exists(p):
+                os.unlink(p)
+    north = None
+    if (G == 8 or args.north_star) and not args.no_north_star:
+        north = run_north_star(args, rank, ws, timer, N=args.ns_n)
 
     timed = max(1, int(k_n))
     avg_ms = k_ms / timed
-    flops_per_launch = k_fl / timed
+    line = assemble_line(args, G, ws, N, T, host, t_roof, terms, bw_src, dod, avg_ms, k_fl / timed, timed,
+                         k_ms, ms_dod, topo, ablation, north, cpu)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+def assemble_line(args, G, ws, N, T, host, t_roof, terms, bw_src, dod, avg_ms, flops_per_launch, timed,
+                  k_ms, ms_dod, topo, ablation=None, north=None, cpu=None):
+    """The one JSON line (pure: tested on CPU by tests/test_bench_line.py)."""
     achieved = flops_per_launch / (avg_ms * 1e-3) / 1e12 if avg_ms > 0 else None
     mode = "rank mode: one process per GPU" if ws > 1 else "one process"
+    grid = "x".join(map(str, _grid(G)))
     roof = {"bound": "tensor", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
             "frac": (achieved / FP64_PEAK_TFLOPS) if achieved else None, "traffic": traffic_from_profiles(T),
             "kernel": "dgemm_tma_kernel (grouped launch; TMA + mbarrier pipeline; FP64 DMMA.8x8x4 via mma.sync.m8n8k4.f64)",
@@ -415,32 +573,42 @@ def run_xk(args, rank, ws):
                            "MEASURED_PEAKS.json); DMMA microbenchmark on this pool measured 37.07",
             "per_launch": "one grouped launch = a batch of tile tasks, 2*T^3 flops each (T=%d); %.3g flops "
                           "per launch on average; %d launches (all GPUs) timed with CUDA events on their kernel "
-                          "stream in a second pass of the same K steps (launches serialised while timed), avg "
-                          "%.3f ms; share of the step: %.3f" % (T, flops_per_launch, timed, avg_ms,
-                                                                k_ms / G / (ms * 1.0))}
-    line = {"metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": G, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+                          "stream in a second pass of the data-on-device steps (launches serialised while "
+                          "timed), avg %.3f ms; share of the data-on-device step: %.3f"
+                          % (T, flops_per_launch, timed, avg_ms, k_ms / G / max(ms_dod, 1e-9))}
+    e2e = {"value": host["wall_tflops"], "unit": "TFLOP/s", "h2d_bytes_per_step": host["h2d"],
+           "d2h_bytes_per_step": host["d2h"], "p2p_bytes_per_step": host["p2p"],
+           "ms_per_step": host["wall_ms"], "roofline_frac": t_roof / (host["wall_ms"] * 1e-3),
+           "clock": "host wall clock from xk_dgemm entry to its return (C coherent on the host), summed "
+                    "over the K calls, max over ranks",
+           "roofline": "max(F/(G*P64), B_h2d/BW_h2d(G), B_d2h/BW_d2h(G), (B_h2d+B_d2h)/BW_duplex(G)[, "
+                       "B_p2p/BW_p2p(G)]) with P64=%.1f TFLOP/s/GPU; BW: %s" % (FP64_PEAK_TFLOPS, bw_src),
+           "roofline_terms_ms": terms}
+    line = {"metric": METRIC, "value": host["tflops"], "unit": "TFLOP/s", "n_gpus": G, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": host["ms"], "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": "DGEMM N=%d (m=n=k), tile %d, NN, alpha=1.5, beta=-0.75, %d GPU(s), grid %s, "
-                                   "heuristics %s%s" % (N, T, G, "x".join(map(str, _grid(G))), args.topo,
-                                                        "+optimistic" if args.optimistic else ""),
+            "config": {"workload": "DGEMM N=%d (m=n=k), tile %d, NN, alpha=1.5, beta=-0.75, host-resident "
+                                   "column-major, %d GPU(s), grid %s, heuristics %s%s"
+                                   % (N, T, G, grid, args.topo, "+optimistic" if args.optimistic else ""),
                        "N": N, "tile": T,
-                       "parallelism": "%s; owner-computes 2D block-cyclic %s" % (mode, "x".join(map(str, _grid(G)))),
-                       "value_mode": "data-on-device: A,B,C resident (prefetched), xk_dgemm_async + xk_sync per step",
-                       "e2e_mode": "xk_dgemm from pinned host memory, all H2D/D2H in the timed region",
-                       "l2": "no flush: each matrix is 8.6 GB >> 126 MB L2",
+                       "parallelism": "%s; owner-computes 2D block-cyclic %s" % (mode, grid),
+                       "value_mode": "end to end (the metric): xk_dgemm from pinned host memory, every "
+                                     "H2D/D2H inside the timed region, C coherent on the host after each "
+                                     "step; CUDA events with a full device synchronize on both sides",
+                       "l2": "no flush: each matrix is %.1f GB >> 126 MB L2" % (8.0 * N * N / 1e9),
                        "inputs": "splitmix64 uniform [-1,1), seeds A=1 B=2 C=3"},
-            "gpu_launches": launches, "clocks": clk, "roofline": roof, "e2e": e2e,
-            "topology_MBps": topo["bw_MBps"], "task_rate_mflops": topo["task_rate_mflops"]}
-    if rank == 0 and not args.no_cpu_baseline and ws == 1:
-        line["cpu_baseline"] = cpu_baseline(N, A, B, C)
-    xk.finalize()
-    barrier(ws)
-    if rank == 0:
-        for p in paths:
-            if os.path.exists(p):
-                os.unlink(p)
-        print(json.dumps(line), flush=True)
+            "gpu_launches": host["launches"], "clocks": host["clocks"], "roofline": roof, "e2e": e2e,
+            "roofline_frac_e2e": t_roof / (host["ms"] * 1e-3),
+            "data_on_device": dod, "h2d_bytes_per_gpu": host["h2d_per_gpu"],
+            "topology_MBps": topo["bw_MBps"], "host_links_all_MBps": topo.get("host_all_MBps"),
+            "task_rate_mflops": topo["task_rate_mflops"]}
+    if ablation is not None:
+        line["ablation"] = ablation
+    if north is not None:
+        line["north_star"] = north
+    if cpu is not None:
+        line["cpu_baseline"] = cpu
+    return line
 
 
 def _grid(G):

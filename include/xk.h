@@ -222,8 +222,25 @@ typedef struct xk_topo {
     int64_t bw_MBps[(XK_MAX_GPUS + 1) * (XK_MAX_GPUS + 1)]; /* row-major, stride ngpus+1 */
     int perf_rank[XK_MAX_GPUS * XK_MAX_GPUS]; /* cuDeviceGetP2PAttribute PERFORMANCE_RANK, logged only (Q6) */
     int64_t task_rate_mflops;                 /* tile-task FP64 rate used by the planner */
+    /* Host links with every GPU copying AT ONCE (xk_probe_host_links; 0 until it ran):
+     * aggregate MB/s over all G GPUs for [0] H2D only, [1] D2H only, [2] full duplex (H2D and
+     * D2H together, total bytes both ways / time).  Host DRAM and the root complexes are shared,
+     * so these bound the PCIe term of the roofline (SecII-B, SecIV-D)
+     * rather than G x the per-GPU entries of bw_MBps. */
+    int64_t host_all_MBps[3];
+    int64_t host_probe_bytes;                 /* bytes per GPU per direction of that probe */
 } xk_topo_t;
 int xk_get_topology(xk_topo_t *out);
+/* Time the host links with all GPUs copying at once (SURVEY.md §8(d) "BW_h2d(G), BW_d2h(G),
+ * full duplex"): every GPU copies bytes_per_gpu between its own pinned host region (distinct
+ * per GPU, allocated here and freed before return) and device memory, H2D only, D2H only,
+ * then both directions together; best of 2 after a warm-up, wall clock around the whole
+ * group (rank mode: barrier-started, each rank's time in the session file, aggregate over
+ * the slowest).  Results in xk_get_topology().host_all_MBps.  Untimed set-up, like the
+ * init probe.  Waits for pending work first.  Rank mode: collective.  Returns
+ * XK_ERR_OOM when neither the pinned host nor the device buffers can be allocated (the size
+ * is halved down to 64 MiB before giving up), XK_ERR_CUDA on a copy failure. */
+int xk_probe_host_links(int64_t bytes_per_gpu);
 
 /* ------------------------------------------------------------------ planner (no GPU) */
 /* The planner is a pure function of (call, topology, flags, directory state): tests run

@@ -235,7 +235,15 @@ def get_topology():
     G = t.ngpus
     bw = [[t.bw_MBps[s * (G + 1) + d] for d in range(G + 1)] for s in range(G + 1)]
     rank = [[t.perf_rank[s * G + d] for d in range(G)] for s in range(G)]
-    return {"ngpus": G, "bw_MBps": bw, "perf_rank": rank, "task_rate_mflops": t.task_rate_mflops}
+    return {"ngpus": G, "bw_MBps": bw, "perf_rank": rank, "task_rate_mflops": t.task_rate_mflops,
+            "host_all_MBps": {"h2d": t.host_all_MBps[0], "d2h": t.host_all_MBps[1],
+                              "duplex": t.host_all_MBps[2]},
+            "host_probe_bytes": t.host_probe_bytes}
+
+
+def probe_host_links(bytes_per_gpu=4 << 30):
+    """xk_probe_host_links: all GPUs copy at once (H2D, D2H, duplex); see get_topology()."""
+    return _check(lib().xk_probe_host_links(int(bytes_per_gpu)))
 
 
 # ---------------------------------------------------------------------------- planner

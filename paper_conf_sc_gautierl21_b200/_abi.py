@@ -54,7 +54,8 @@ class Stats(ctypes.Structure):
 
 class Topo(ctypes.Structure):
     _fields_ = [("ngpus", c_int), ("bw_MBps", i64 * ((MAX_GPUS + 1) * (MAX_GPUS + 1))),
-                ("perf_rank", c_int * (MAX_GPUS * MAX_GPUS)), ("task_rate_mflops", i64)]
+                ("perf_rank", c_int * (MAX_GPUS * MAX_GPUS)), ("task_rate_mflops", i64),
+                ("host_all_MBps", i64 * 3), ("host_probe_bytes", i64)]
 
 
 class Flags(ctypes.Structure):
@@ -119,6 +120,7 @@ _SIGS = [
     ("xk_reset_stats", c_int, []),
     ("xk_set_kernel_timing", c_int, [c_int]),
     ("xk_get_topology", c_int, [ctypes.POINTER(Topo)]),
+    ("xk_probe_host_links", c_int, [i64]),
     ("xk_trace", c_int, [ctypes.c_char_p]),
     ("xk_plan_session_create", c_int, [ctypes.POINTER(Topo), ctypes.POINTER(Flags), ctypes.POINTER(vp)]),
     ("xk_plan_session_call", c_int, [vp, ctypes.POINTER(Call), ctypes.POINTER(PlanRec), i64,

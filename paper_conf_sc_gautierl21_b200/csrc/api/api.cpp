@@ -403,7 +403,16 @@ int xk_get_topology(xk_topo_t *out) {
     for (int s = 0; s < G; ++s)
         for (int d = 0; d < G; ++d) out->perf_rank[s * G + d] = rt->perf_rank[(size_t)s * G + d];
     out->task_rate_mflops = rt->topo.rate_mflops;
+    for (int q = 0; q < 3; ++q) out->host_all_MBps[q] = rt->host_all_MBps[q];
+    out->host_probe_bytes = rt->host_probe_bytes;
     return XK_OK;
+}
+
+int xk_probe_host_links(int64_t bytes_per_gpu) {
+    xk::Runtime *rt = runtime();
+    if (!rt) return need_init();
+    if (bytes_per_gpu <= 0) return XK_ERR_CONFIG;
+    return rt->probe_host_links(bytes_per_gpu);
 }
 
 }  // extern "C"

@@ -91,6 +91,9 @@ public:
     int sync_all();
     int invalidate(uint64_t base, int64_t m, int64_t n, int64_t ld);
 
+    int probe_host_links(int64_t bytes_per_gpu);  // SURVEY §8(d) concurrent BW_h2d/d2h/duplex
+    int64_t host_all_MBps[3] = {0, 0, 0};
+    int64_t host_probe_bytes = 0;
     int register_host(void *p, size_t bytes);
     int unregister_host(void *p);
     int ensure_pinned(uint64_t base, int64_t rows, int64_t cols, int64_t ld);

@@ -35,6 +35,8 @@ struct SessionRank {
     int64_t bw_local;              // bw[rank][rank]
     int64_t rate_mflops;           // FP64 tile-task rate (rank 0's is used)
     uint64_t plan_cfg;             // hash of the plan-shaping configuration (must agree)
+    double host_probe_ms;          // xk_probe_host_links: this rank's time for one pattern
+    int64_t host_probe_bytes;      // ... and the bytes it moved
 };
 
 struct SessionHeader {

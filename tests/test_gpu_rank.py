@@ -152,3 +152,50 @@ def test_rank_mode_refuses_diverging_configuration():
     different plans: xk_init fails with XK_ERR_CONFIG on every rank, nobody hangs."""
     outs = run_ranks(2, "mismatch", 512, 128, timeout=300)
     assert [o["init_error"] for o in outs] == [4, 4]
+
+
+def test_bench_under_torchrun_emits_round2_keys():
+    """bench.py under torchrun (2 ranks on the box's GPU(s), rank mode): one JSON line with the
+    host-resident value, e2e (with the concurrent-probe roofline), data_on_device, the
+    heuristic ablation (every mode, per-GPU H2D bytes) and the north-star block (forced at
+    G = 2, small N to stay quick)."""
+    env = dict(os.environ, XK_DIST_BACKEND="gloo")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", "29631", os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--n", "16384", "--tile", "2048", "--steps", "1", "--warmup", "1",
+           "--no-cpu-baseline", "--north-star", "--ns-n", "8192", "--host-probe-mib", "256"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    line = json.loads([ln for ln in r.stdout.splitlines() if ln.startswith("{")][-1])
+    assert line["n_gpus"] == 2 and line["value"] > 0 and line["gpu_launches"] > 0
+    assert line["e2e"]["h2d_bytes_per_step"] == 3 * 8 * 16384 ** 2
+    assert line["host_links_all_MBps"]["h2d"] > 0 and line["host_links_all_MBps"]["duplex"] > 0
+    assert line["data_on_device"]["value"] > 0
+    abl = line["ablation"]
+    for mode in ("full", "no_optimistic", "no_optimistic_no_topo", "home"):
+        assert abl[mode]["tflops"] > 0 and len(abl[mode]["h2d_bytes_per_gpu"]) == 2
+    # closed forms (SURVEY App. B) at N=16384, T=2048 on the 2x1 grid: FULL reads A, B, C once
+    # (6.44 GB), HOME reads every A row tile once per requesting GPU (r_A = min(Q, t) = 1) and
+    # every B column tile once per grid row (r_B = min(P, t) = 2)
+    tile = 8 * 2048 * 2048
+    assert abl["full"]["h2d_bytes"] == 3 * 64 * tile
+    assert abl["home"]["h2d_bytes"] == (8 * 8 * 1 + 8 * 8 * 2 + 64) * tile
+    assert line["north_star"]["tflops"] > 0
+
+
+def test_probe_host_links_single_process():
+    """xk_probe_host_links: all GPUs copying at once; one GPU and 2 logical GPUs (which share
+    one physical link, so the aggregate stays near one link's bandwidth)."""
+    from tests.gpu_util import device_map
+    for G in (1, 2):
+        xk.init(ngpus=G, phys=device_map(G), probe=True, tile=512)
+        try:
+            assert xk.probe_host_links(256 << 20) == 0
+            t = xk.get_topology()
+        finally:
+            xk.finalize()
+        ha = t["host_all_MBps"]
+        single = t["bw_MBps"][G][0]
+        assert t["host_probe_bytes"] == 256 << 20
+        assert ha["h2d"] > 0.5 * single and ha["d2h"] > 0 and ha["duplex"] > 0
+        assert ha["h2d"] < 1.5 * G * single
