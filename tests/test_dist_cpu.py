@@ -25,14 +25,16 @@ assert mx == 11.0, mx
 assert bench.sum_over_ranks([1.0 + rank, 5.0], ws) == [3.0, 10.0]
 # rank-mode host matrices: one generator run on rank 0, the same bits on every rank
 import numpy as np, inputs
-A, B, C, paths = bench.share_inputs(48, rank, ws)
+A, B, C, paths, base = bench.share_inputs(48, rank, ws)
 assert np.array_equal(np.asarray(B), inputs.uniform(inputs.SEED_B, 48, 48))
 assert A.shape == (48, 48) and np.asfortranarray(A).flags.f_contiguous
-assert paths[-1].endswith(".session")
-assert len(set(paths)) == (1 if os.environ.get("XK_SHARE") == "memfd" else 4)
+assert base and base.startswith(("/dev/shm", "/tmp"))  # session files: base + ".session<n>"
+assert len(paths) == (0 if os.environ.get("XK_SHARE") == "memfd" else 3)
+# per-GPU values gathered in rank order (per-GPU H2D bytes of the ablation)
+assert bench.gather_per_gpu(7.0 + rank, ws) == [7.0, 8.0]
 bench.barrier(ws)
 if rank == 0:
-    for p in paths[:-1]:
+    for p in paths:
         os.unlink(p)
 # reference arm under torchrun: rank 0 alone prints one JSON line, the other exits quietly
 if rank == 0:
