@@ -290,6 +290,67 @@ void Planner::emit_d2h(int key, int src, int64_t r0, int64_t c0, int64_t rows, i
     }
 }
 
+// R16 quotas: split count[S] host tiles of each shared requester set S over its members so
+// that the largest per-GPU total (forced[g] + assigned) is as small as possible.  Binary
+// search on that maximum L; feasibility is a max-flow (source -> set S, capacity count[S];
+// S -> member g; g -> sink, capacity L - forced[g]) by Edmonds-Karp: BFS over nodes in index
+// order (0 source, 1..nS sets, then GPUs, then sink), augmenting by the bottleneck.  The flow
+// on S -> g is the quota (deterministic; the CPU plan model runs the same procedure).
+static std::vector<std::vector<int64_t>> balance_quotas(int G, const std::vector<uint32_t> &sets,
+                                                        const std::vector<int64_t> &count,
+                                                        const std::vector<int64_t> &forced) {
+    const int nS = (int)sets.size(), V = nS + G + 2, src = 0, snk = V - 1;
+    int64_t total = 0, fmax = 0, ftot = 0;
+    for (int64_t c : count) total += c;
+    for (int64_t f : forced) { fmax = std::max(fmax, f); ftot += f; }
+    std::vector<int64_t> cap, flow;
+    auto run = [&](int64_t L) {
+        cap.assign((size_t)V * V, 0);
+        flow.assign((size_t)V * V, 0);
+        for (int i = 0; i < nS; ++i) {
+            cap[(size_t)src * V + 1 + i] = count[i];
+            for (int g = 0; g < G; ++g)
+                if (sets[i] >> g & 1) cap[(size_t)(1 + i) * V + 1 + nS + g] = total;
+        }
+        for (int g = 0; g < G; ++g) cap[(size_t)(1 + nS + g) * V + snk] = std::max<int64_t>(0, L - forced[g]);
+        int64_t got = 0;
+        std::vector<int> par(V);
+        for (;;) {
+            std::fill(par.begin(), par.end(), -1);
+            par[src] = src;
+            std::vector<int> q{src};
+            for (size_t h = 0; h < q.size() && par[snk] < 0; ++h) {
+                const int u = q[h];
+                for (int v = 0; v < V; ++v)
+                    if (par[v] < 0 && cap[(size_t)u * V + v] - flow[(size_t)u * V + v] > 0) {
+                        par[v] = u;
+                        q.push_back(v);
+                    }
+            }
+            if (par[snk] < 0) break;
+            int64_t b = INT64_MAX;
+            for (int v = snk; v != src; v = par[v])
+                b = std::min(b, cap[(size_t)par[v] * V + v] - flow[(size_t)par[v] * V + v]);
+            for (int v = snk; v != src; v = par[v]) {
+                flow[(size_t)par[v] * V + v] += b;
+                flow[(size_t)v * V + par[v]] -= b;
+            }
+            got += b;
+        }
+        return got == total;
+    };
+    int64_t lo = std::max(fmax, (total + ftot + G - 1) / G), hi = fmax + total;
+    while (lo < hi) {
+        const int64_t mid = lo + (hi - lo) / 2;
+        if (run(mid)) hi = mid; else lo = mid + 1;
+    }
+    run(lo);
+    std::vector<std::vector<int64_t>> quota(nS, std::vector<int64_t>(G, 0));
+    for (int i = 0; i < nS; ++i)
+        for (int g = 0; g < G; ++g) quota[i][g] = std::max<int64_t>(0, flow[(size_t)(1 + i) * V + 1 + nS + g]);
+    return quota;
+}
+
 // steps 2, 3, 6, 7: per-GPU lists ordered by the generator's sort key (k-major, k-shifted
 // anti-diagonal), event loop on the smallest request time, task timing, output
 // versioning, D2H after the last writer of each output tile.
@@ -323,6 +384,72 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
         for (auto &t : tasks) {
             auto it = slot.find({t.out_key, t.out_ver - 1});
             t.war = (it == slot.end()) ? -1 : it->second;
+        }
+    }
+    // Balance-aware first host pull (reading R16; FULL mode only: it forwards from an in-flight
+    // copy).  An input tile version valid only on the host at the start of the call crosses
+    // PCIe once; which requester's link carries it is fixed here, before the event loop, so that
+    // the most loaded host link carries as few tiles as possible: a tile read by one GPU goes to
+    // that GPU; the tiles read by several GPUs are grouped by requester set and split by the
+    // min-max quotas of balance_quotas(), then dealt inside each set in first-appearance order
+    // to the member furthest below its quota.  When another requester asks first, the tile is
+    // pulled to its designated GPU and forwarded from there (store-and-forward over NVLink).
+    std::vector<int> puller(pending.size(), -1);
+    if (flags_.optimistic && flags_.topo != XK_TOPO_HOME && G > 1) {
+        std::vector<uint32_t> mask(pending.size(), 0);
+        std::vector<int> order;  // slots in first-appearance order
+        std::vector<int> slot_key(pending.size(), -1);
+        std::vector<int64_t> slot_ver(pending.size(), 0);
+        for (const auto &t : tasks)
+            for (const auto &in : t.in) {
+                if (slot_key[in.cnt] < 0) order.push_back(in.cnt);
+                mask[in.cnt] |= 1u << t.gpu;
+                slot_key[in.cnt] = in.key;
+                slot_ver[in.cnt] = in.ver;
+            }
+        auto host_only = [&](int s) {
+            const Entry &e = entries_[slot_key[s]];
+            if (e.ver != slot_ver[s] || !(e.host.present && e.host.ver == e.ver)) return false;
+            for (const NodeCopy &g : e.gpu)
+                if (g.present && g.ver == e.ver) return false;
+            return true;
+        };
+        std::vector<int64_t> forced(G, 0);
+        std::vector<uint32_t> sets;            // shared requester sets, first-appearance order
+        std::vector<int64_t> count;            // host-only tiles per set
+        std::unordered_map<uint32_t, int> set_id;
+        for (int s : order) {
+            if (!host_only(s)) continue;
+            if ((mask[s] & (mask[s] - 1)) == 0) {
+                int g = __builtin_ctz(mask[s]);
+                puller[s] = g;
+                forced[g]++;
+                continue;
+            }
+            auto it = set_id.find(mask[s]);
+            if (it == set_id.end()) {
+                it = set_id.emplace(mask[s], (int)sets.size()).first;
+                sets.push_back(mask[s]);
+                count.push_back(0);
+            }
+            count[it->second]++;
+        }
+        if (!sets.empty()) {
+            std::vector<std::vector<int64_t>> quota = balance_quotas(G, sets, count, forced);
+            std::vector<std::vector<int64_t>> given(sets.size(), std::vector<int64_t>(G, 0));
+            for (int s : order) {
+                if (puller[s] >= 0 || !host_only(s)) continue;
+                const int id = set_id[mask[s]];
+                const auto &q = quota[id];
+                auto &a = given[id];
+                int best = -1;  // least a/q among members with quota left (ties: lowest id)
+                for (int g = 0; g < G; ++g) {
+                    if (!(mask[s] >> g & 1) || a[g] >= q[g]) continue;
+                    if (best < 0 || a[g] * q[best] < a[best] * q[g]) best = g;
+                }
+                a[best]++;
+                puller[s] = best;
+            }
         }
     }
     // last writer per output tile
@@ -388,6 +515,16 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
         for (size_t p = 0; p < t.in.size(); ++p) {
             const Input &in = t.in[p];
             Entry &e = entries_[in.key];
+            const int pl = puller[in.cnt];
+            if (pl >= 0 && pl != d && !(e.gpu[d].present && e.gpu[d].ver == in.ver)) {
+                // R16: the first host read of this tile goes to its designated GPU
+                bool any = false;
+                for (const NodeCopy &g : e.gpu) any = any || (g.present && g.ver == in.ver);
+                if (!any && !emit_copy(in.key, in.ver, pl, treq, in.operand, out)) {
+                    err = "no valid copy of an input tile (invalidated without coherence?)";
+                    return XK_ERR_INTERNAL;
+                }
+            }
             if (!(e.gpu[d].present && e.gpu[d].ver == in.ver) &&
                 !emit_copy(in.key, in.ver, d, treq, in.operand, out)) {
                 err = "no valid copy of an input tile (invalidated without coherence?)";

@@ -45,6 +45,61 @@ def near_square(G):
     return G // q, q
 
 
+def min_max_quotas(G, sets, count, forced):
+    """R16: split count[i] tiles of requester set sets[i] over its members minimising the
+    largest forced[g] + assigned[g]: binary search on that maximum, feasibility by max-flow
+    (Edmonds-Karp, BFS in node order: source, sets, GPUs, sink).  Returns the flows set -> GPU."""
+    nS = len(sets)
+    V, src, snk = nS + G + 2, 0, nS + G + 1
+    total = sum(count)
+
+    def run(L):
+        cap = [[0] * V for _ in range(V)]
+        flow = [[0] * V for _ in range(V)]
+        for i, S in enumerate(sets):
+            cap[src][1 + i] = count[i]
+            for g in S:
+                cap[1 + i][1 + nS + g] = total
+        for g in range(G):
+            cap[1 + nS + g][snk] = max(0, L - forced[g])
+        got = 0
+        while True:
+            par = [-1] * V
+            par[src] = src
+            q = [src]
+            h = 0
+            while h < len(q) and par[snk] < 0:
+                u = q[h]
+                h += 1
+                for v in range(V):
+                    if par[v] < 0 and cap[u][v] - flow[u][v] > 0:
+                        par[v] = u
+                        q.append(v)
+            if par[snk] < 0:
+                break
+            b, v = None, snk
+            while v != src:
+                r = cap[par[v]][v] - flow[par[v]][v]
+                b = r if b is None else min(b, r)
+                v = par[v]
+            v = snk
+            while v != src:
+                flow[par[v]][v] += b
+                flow[v][par[v]] -= b
+                v = par[v]
+            got += b
+        return got == total, flow
+    lo, hi = max(max(forced), -(-(total + sum(forced)) // G)), max(forced) + total
+    while lo < hi:
+        mid = (lo + hi) // 2
+        if run(mid)[0]:
+            hi = mid
+        else:
+            lo = mid + 1
+    flow = run(lo)[1]
+    return [[max(0, flow[1 + i][1 + nS + g]) for g in range(G)] for i in range(nS)]
+
+
 class Copy:
     __slots__ = ("ver", "t_done", "producer", "depth")
 
@@ -524,6 +579,49 @@ class Model:
                 last[o] = t
         for t in last.values():
             t["last"] = True
+        # R16 balance-aware first host pull (FULL mode): who carries each host-only input
+        puller = {}
+        if self.opt and self.mode != HOME and self.G > 1:
+            req, order = {}, []
+            for t in tasks:
+                for (tl, v, _) in t["ins"]:
+                    key = (id(tl), v)
+                    if key not in req:
+                        req[key] = (tl, v, set())
+                        order.append(key)
+                    req[key][2].add(t["gpu"])
+            forced = [0] * self.G
+            sets, count = [], {}
+            shared = []
+            for key in order:
+                tl, v, gs = req[key]
+                if not (tl.ver == v and tl.host is not None and tl.host.ver == v
+                        and not any(c.ver == v for c in tl.gpus.values())):
+                    continue
+                if len(gs) == 1:
+                    (g,) = gs
+                    puller[key] = g
+                    forced[g] += 1
+                    continue
+                fs = frozenset(gs)
+                if fs not in count:
+                    sets.append(fs)
+                    count[fs] = 0
+                count[fs] += 1
+                shared.append(key)
+            if sets:
+                quota = min_max_quotas(self.G, sets, [count[s] for s in sets], forced)
+                given = {s: [0] * self.G for s in sets}
+                for key in shared:
+                    gs = frozenset(req[key][2])
+                    q, a = quota[sets.index(gs)], given[gs]
+                    cands = [g for g in sorted(gs) if a[g] < q[g]]
+                    best = cands[0]
+                    for g in cands[1:]:
+                        if a[g] * q[best] < a[best] * q[g]:
+                            best = g
+                    a[best] += 1
+                    puller[key] = best
         lists = [[] for _ in range(self.G)]
         for t in tasks:
             lists[t["gpu"]].append(t)
@@ -558,6 +656,10 @@ class Model:
             ready_at = 0
             for p, (tl, v, operand) in enumerate(t["ins"]):
                 c = tl.gpus.get(d)
+                pl = puller.get((id(tl), v))
+                if (pl is not None and pl != d and (c is None or c.ver != v)
+                        and not any(x.ver == v for x in tl.gpus.values())):
+                    self.copy_in(tl, v, pl, treq, operand, out)  # first host read to its GPU
                 if c is None or c.ver != v:
                     self.copy_in(tl, v, d, treq, operand, out)
                 c = tl.gpus[d]

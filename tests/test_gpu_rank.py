@@ -162,7 +162,7 @@ def test_bench_under_torchrun_emits_round2_keys():
     env = dict(os.environ, XK_DIST_BACKEND="gloo")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", "29631", os.path.join(ROOT, "bench.py"),
-           "--gpus", "2", "--n", "16384", "--tile", "2048", "--steps", "1", "--warmup", "1",
+           "--gpus", "2", "--size", "16384", "--tile", "2048", "--steps", "1", "--warmup", "1",
            "--no-cpu-baseline", "--north-star", "--ns-n", "8192", "--host-probe-mib", "256"]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
     assert r.returncode == 0, r.stderr[-3000:]
