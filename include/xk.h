@@ -202,6 +202,10 @@ typedef struct xk_stats {
                                         column = destination, stride ngpus+1, index ngpus = host */
     double trace_ms[4];              /* with tracing on: summed op time by kind
                                         [H2D, P2P, kernel, D2H] (paper Fig. 6 breakdown) */
+    int64_t plan_records;            /* plan records produced (every GPU's) */
+    int64_t plan_records_local;      /* ... of which executed by this process (rank mode: its GPU) */
+    double host_issue_ms;            /* host wall time planning + issuing them (the per-call
+                                        "creation and scheduling of dynamic tasks") */
 } xk_stats_t;
 int xk_get_stats(xk_stats_t *out);
 int xk_reset_stats(void);

@@ -49,7 +49,8 @@ class Stats(ctypes.Structure):
                 ("host_registrations", i64), ("kernel_ms_total", c_double),
                 ("kernel_timed_launches", i64), ("kernel_timed_flops", i64),
                 ("link_bytes", i64 * ((MAX_GPUS + 1) * (MAX_GPUS + 1))),
-                ("trace_ms", c_double * 4)]
+                ("trace_ms", c_double * 4), ("plan_records", i64), ("plan_records_local", i64),
+                ("host_issue_ms", c_double)]
 
 
 class Topo(ctypes.Structure):

@@ -1554,7 +1554,12 @@ int Runtime::run_impl(const xk_call_t &call, bool wait) {
     std::fill(batches_in_call_.begin(), batches_in_call_.end(), 0);
     // records are issued as the planner produces them: the GPUs start on the first copies
     // and tasks while the rest of the call is still being planned
-    Planner::Sink sink = [this](const Rec &r) { return issue(r); };
+    Planner::Sink sink = [this](const Rec &r) {
+        stats.plan_records++;
+        if (here(r.r)) stats.plan_records_local++;
+        return issue(r);
+    };
+    const auto t_issue = std::chrono::steady_clock::now();
     rc = planner_->plan(call, recs, err, &sink);
     if (rc) {
         if (rc != XK_ERR_CUDA && rc != XK_ERR_OOM) set_error(err);
@@ -1562,6 +1567,7 @@ int Runtime::run_impl(const xk_call_t &call, bool wait) {
     }
     for (size_t g = 0; g < batch_.size(); ++g)
         if ((rc = flush_batch((int)g))) return rc;
+    stats.host_issue_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_issue).count();
     if (call.routine == XK_ROUTINE_SYNC) {
         // xk_sync: everything issued has completed (the API synchronised first), so tiles the
         // planner dropped -- e.g. a call's shadow copies of C -- can go back to the pool

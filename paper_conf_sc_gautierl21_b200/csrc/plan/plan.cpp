@@ -357,33 +357,26 @@ static std::vector<std::vector<int64_t>> balance_quotas(int G, const std::vector
 int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &out, std::string &err) {
     const int G = topo_.G;
     const int W = std::max(1, flags_.window);
-    // pending reads per (key, version) in this call; last writer per output tile
-    struct PairHash {
-        size_t operator()(const std::pair<int, int64_t> &p) const {
-            return std::hash<uint64_t>()(((uint64_t)p.first << 32) ^ (uint64_t)p.second * 0x9E3779B97F4A7C15ULL);
-        }
-    };
-    // pending reads per (key, version) in this call, resolved once to flat counter slots
+    // pending reads per (key, version) in this call, resolved once to flat counter slots.
+    // Tasks are in program order and a key's versions only grow along it, so all reads of
+    // (key, v) precede the write of v + 1: one (version, slot) pair per key suffices.
     std::vector<int64_t> pending;
     {
-        std::unordered_map<std::pair<int, int64_t>, int, PairHash> slot;
-        slot.reserve(tasks.size() * 2 + 16);
-        auto slot_of = [&](int key, int64_t ver) {
-            auto it = slot.find({key, ver});
-            if (it != slot.end()) return it->second;
-            int id = (int)pending.size();
-            pending.push_back(0);
-            slot.emplace(std::make_pair(key, ver), id);
-            return id;
-        };
-        for (auto &t : tasks)
+        std::vector<int64_t> last_ver(entries_.size(), -1);
+        std::vector<int> last_slot(entries_.size(), -1);
+        pending.reserve(tasks.size());
+        for (auto &t : tasks) {
             for (auto &in : t.in) {
-                in.cnt = slot_of(in.key, in.ver);
+                if (last_slot[in.key] < 0 || last_ver[in.key] != in.ver) {
+                    last_ver[in.key] = in.ver;
+                    last_slot[in.key] = (int)pending.size();
+                    pending.push_back(0);
+                }
+                in.cnt = last_slot[in.key];
                 pending[in.cnt]++;
             }
-        for (auto &t : tasks) {
-            auto it = slot.find({t.out_key, t.out_ver - 1});
-            t.war = (it == slot.end()) ? -1 : it->second;
+            // WAR: readers of the version this task overwrites (all precede it)
+            t.war = (last_slot[t.out_key] >= 0 && last_ver[t.out_key] == t.out_ver - 1) ? last_slot[t.out_key] : -1;
         }
     }
     // Balance-aware first host pull (reading R16; FULL mode only: it forwards from an in-flight

@@ -166,11 +166,18 @@ private:
         int64_t skey[5] = {0, 0, 0, 0, 0};  // per-GPU list order
     };
     // symbolic versions while a call's task list is generated (program order)
-    struct Versions {
-        std::unordered_map<int, int64_t> cur;
+    struct Versions {  // flat by directory id: -1 = not written yet in this call
+        std::vector<int64_t> cur;
         const std::vector<Entry> *e = nullptr;
-        int64_t get(int key) { auto it = cur.find(key); return it == cur.end() ? (*e)[key].ver : it->second; }
-        int64_t bump(int key) { int64_t v = get(key) + 1; cur[key] = v; return v; }
+        int64_t get(int key) const {
+            return ((size_t)key < cur.size() && cur[key] >= 0) ? cur[key] : (*e)[key].ver;
+        }
+        int64_t bump(int key) {
+            const int64_t v = get(key) + 1;
+            if ((size_t)key >= cur.size()) cur.resize(std::max(e->size(), (size_t)key + 1), -1);
+            cur[key] = v;
+            return v;
+        }
     };
 
     int plan_impl(const xk_call_t &c, std::vector<Rec> &out, std::string &err);
