@@ -208,6 +208,32 @@ def test_full_size_n16384_exact_freivalds():
         assert np.array_equal(lhs, rhs)
 
 
+@pytest.mark.parametrize("T", [2048, 4096])
+def test_eight_logical_gpus_full_tiles_exact(T):
+    """8 logical GPUs (4x2 grid, the north-star layout) at the bench's tile sizes, N=16384,
+    exact-integer inputs: 4096 sampled entries bitwise equal to the oracle's dot loop (every
+    summation order is exact here) and an exact Freivalds check of the whole C."""
+    N = 16384
+    A, B, C0 = inputs.integers(1, N, N), inputs.integers(2, N, N), inputs.integers(3, N, N)
+    C = C0.copy(order="F")
+    logical(8, tile=T)
+    try:
+        xk.register(A); xk.register(B); xk.register(C)
+        xk.reset_stats()
+        assert xk.dgemm("N", "N", N, N, N, 2.0, A, N, B, N, -1.0, C, N) == 0
+        st = xk.get_stats()
+    finally:
+        xk.finalize()
+    t = N // T
+    assert sum(st["tasks"]) == t ** 3 and all(x > 0 for x in st["tasks"])
+    rng = np.random.default_rng(11)
+    ii = rng.integers(0, N, 4096); jj = rng.integers(0, N, 4096)
+    ref = oracle.dgemm_sampled("N", "N", N, 2.0, A, B, -1.0, C0[ii, jj], ii, jj)
+    assert np.array_equal(C[ii, jj], ref)
+    x = rng.integers(-4, 5, N).astype(np.float64)
+    assert np.array_equal(C @ x, 2.0 * (A @ (B @ x)) - 1.0 * (C0 @ x))
+
+
 @pytest.mark.parametrize("N,T", [(32768, 4096), (32768, 2048), (65536, 4096)])
 def test_full_size_sampled(N, T):
     """The bench workload (N=32768, T=4096 -- bench.py's launch configuration -- and T=2048)

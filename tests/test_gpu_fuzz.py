@@ -101,5 +101,18 @@ def test_random_calls(seed):
                     assert np.all(X == 0)
                     continue
                 assert np.linalg.norm(X - ref) <= 1e-13 * max(np.linalg.norm(ref), 1e-300)
+                # elementwise (Q13): TRMM vs the oracle, |alpha| 4 ka 2^-53 |op(T)||B0|;
+                # TRSM: the componentwise residual of the GPU solution
+                Tm = np.where(tri_mask(ka, uplo == "L"), np.nan_to_num(L, nan=0.0), 0.0)
+                if dg == "U":
+                    Tm[np.diag_indices(ka)] = 1.0
+                opT = Tm.T if ta == "T" else Tm
+                if routine == "trmm":
+                    mag = (np.abs(opT) @ np.abs(B0)) if side == "L" else (np.abs(B0) @ np.abs(opT))
+                    assert np.all(np.abs(X - ref) <= 4 * ka * 2.0 ** -53 * abs(alpha) * mag)
+                else:
+                    R = (opT @ X - alpha * B0) if side == "L" else (X @ opT - alpha * B0)
+                    magr = (np.abs(opT) @ np.abs(X)) if side == "L" else (np.abs(X) @ np.abs(opT))
+                    assert np.all(np.abs(R) <= 4 * ka * 2.0 ** -53 * (magr + abs(alpha) * np.abs(B0)) * 1.0000001)
     finally:
         xk.finalize()
