@@ -111,6 +111,9 @@ typedef struct xk_config {
 void xk_config_default(xk_config_t *cfg);
 
 /* ------------------------------------------------------------------ lifecycle */
+/* xk_init: set up the GPUs, streams and the planner; with cfg->probe, time the (G+1)^2 link
+ * matrix "during the library initialization" (SecIII-B).  Errors: XK_ERR_CONFIG
+ * (bad grid / topo / ngpus), XK_ERR_NO_DEVICE, XK_ERR_CUDA, XK_ERR_OOM (rank-mode arena). */
 int xk_init(const xk_config_t *cfg); /* NULL -> xk_config_default(); probes topology */
 int xk_finalize(void);               /* waits, frees every device copy, destroys streams */
 int xk_register(void *p, size_t bytes);   /* cudaHostRegister(Portable) once, all GPUs */
@@ -118,7 +121,18 @@ int xk_unregister(void *p);
 const char *xk_last_error(void);
 
 /* ------------------------------------------------------------------ BLAS-3 (FP64) */
-/* C <- alpha*op(A)*op(B) + beta*C ; op(X) = X ('N') or X^T ('T'/'C').
+/* The six routines of the paper's report (SecI, Fig. 5, SecIV-D
+ * P:834-835), each the operation the BLAS standard defines (ref. [1], P:66-67 and
+ * P:1187-1188; argument order and XERBLA numbering as in the reference BLAS), computed by
+ * PLASMA-style tiled algorithms on LAPACK-layout views (SecIII).  The synchronous
+ * form returns with the output coherent on the host; the _async form is the paper's
+ * xkblas_*_async (SecIV-F): it returns once the work is issued and composes with
+ * later calls through the tile cache.  Only the arguments' referenced parts are read
+ * (BLAS "not referenced" rules, header comment above).  Errors: -i for argument i, or a
+ * positive XK_ERR_*.
+ *
+ * DGEMM (Fig. 3, Table II):
+ * C <- alpha*op(A)*op(B) + beta*C ; op(X) = X ('N') or X^T ('T'/'C').
  * A is m x k ('N') or k x m ('T') with lda >= max(1, rows); B is k x n or n x k; C m x n.
  * Errors: -1 transA, -2 transB, -3 m, -4 n, -5 k, -8 lda, -10 ldb, -13 ldc. */
 int xk_dgemm(char transA, char transB, int64_t m, int64_t n, int64_t k, double alpha,
@@ -128,14 +142,16 @@ int xk_dgemm_async(char transA, char transB, int64_t m, int64_t n, int64_t k, do
                    const double *A, int64_t lda, const double *B, int64_t ldb,
                    double beta, double *C, int64_t ldc);
 
-/* C <- alpha*op(A)*op(A)^T + beta*C on the uplo triangle only (op(A) n x k).
+/* DSYRK (SecIV-D):
+ * C <- alpha*op(A)*op(A)^T + beta*C on the uplo triangle only (op(A) n x k).
  * Errors: -1 uplo, -2 trans, -3 n, -4 k, -7 lda, -10 ldc. */
 int xk_dsyrk(char uplo, char trans, int64_t n, int64_t k, double alpha,
              const double *A, int64_t lda, double beta, double *C, int64_t ldc);
 int xk_dsyrk_async(char uplo, char trans, int64_t n, int64_t k, double alpha,
                    const double *A, int64_t lda, double beta, double *C, int64_t ldc);
 
-/* C <- alpha*op(A)*op(B)^T + alpha*op(B)*op(A)^T + beta*C, uplo triangle only.
+/* DSYR2K (Fig. 3):
+ * C <- alpha*op(A)*op(B)^T + alpha*op(B)*op(A)^T + beta*C, uplo triangle only.
  * Errors: -1 uplo, -2 trans, -3 n, -4 k, -7 lda, -9 ldb, -12 ldc. */
 int xk_dsyr2k(char uplo, char trans, int64_t n, int64_t k, double alpha,
               const double *A, int64_t lda, const double *B, int64_t ldb,
@@ -144,7 +160,7 @@ int xk_dsyr2k_async(char uplo, char trans, int64_t n, int64_t k, double alpha,
                     const double *A, int64_t lda, const double *B, int64_t ldb,
                     double beta, double *C, int64_t ldc);
 
-/* C <- alpha*sym(A)*B + beta*C ('L') or alpha*B*sym(A) + beta*C ('R'); only the uplo
+/* DSYMM: C <- alpha*sym(A)*B + beta*C ('L') or alpha*B*sym(A) + beta*C ('R'); only the uplo
  * triangle of A is read.  Errors: -1 side, -2 uplo, -3 m, -4 n, -7 lda, -9 ldb, -12 ldc. */
 int xk_dsymm(char side, char uplo, int64_t m, int64_t n, double alpha,
              const double *A, int64_t lda, const double *B, int64_t ldb,
@@ -153,14 +169,16 @@ int xk_dsymm_async(char side, char uplo, int64_t m, int64_t n, double alpha,
                    const double *A, int64_t lda, const double *B, int64_t ldb,
                    double beta, double *C, int64_t ldc);
 
-/* B <- alpha*op(A)*B ('L') or alpha*B*op(A) ('R'), A triangular (uplo), diag 'U' = unit.
+/* DTRMM: B <- alpha*op(A)*B ('L') or alpha*B*op(A) ('R'), A triangular
+ * (uplo), diag 'U' = unit.
  * Errors: -1 side, -2 uplo, -3 transA, -4 diag, -5 m, -6 n, -9 lda, -11 ldb. */
 int xk_dtrmm(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
              double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
 int xk_dtrmm_async(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
                    double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
 
-/* Solve op(A)*X = alpha*B ('L') or X*op(A) = alpha*B ('R'); B <- X.  Same errors as TRMM. */
+/* DTRSM (Fig. 3, Table II; composed with DGEMM in SecIV-F):
+ * solve op(A)*X = alpha*B ('L') or X*op(A) = alpha*B ('R'); B <- X.  Same errors as TRMM. */
 int xk_dtrsm(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
              double alpha, const double *A, int64_t lda, double *B, int64_t ldb);
 int xk_dtrsm_async(char side, char uplo, char transA, char diag, int64_t m, int64_t n,
@@ -207,6 +225,9 @@ typedef struct xk_stats {
     double host_issue_ms;            /* host wall time planning + issuing them (the per-call
                                         "creation and scheduling of dynamic tasks") */
 } xk_stats_t;
+/* Counters since xk_init / the last xk_reset_stats: the per-link byte counts are the paper's
+ * transfer breakdown (SecIV-E) and the evidence that the heuristics cut PCIe bytes
+ * (P:181-183).  Errors: XK_ERR_NOT_INITIALIZED, XK_ERR_CONFIG (out == NULL). */
 int xk_get_stats(xk_stats_t *out);
 int xk_reset_stats(void);
 /* 1 = time every tile-kernel launch with CUDA events (bench roofline); grouped launches are

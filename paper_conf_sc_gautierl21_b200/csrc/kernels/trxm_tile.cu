@@ -4,10 +4,11 @@
 //
 // TRSM/TRMM tile (PLASMA's dtrsm/dtrmm on a tile): recursive blocking on the
 // order of the triangular matrix -- the two half-size triangles recurse, the off-diagonal
-// block is one GEMM on the sm_100a DMMA tile kernel (dgemm_tile.cu), and below 64 a base
-// kernel solves (or multiplies) one vector per thread, held in registers, against the small
-// triangle held in shared memory (128 vectors per CTA share one triangle load).  Recursive blocking keeps the substitution backward stable (no explicit
-// inverse), so the componentwise residual bound of DESIGN.md reading Q13 holds.
+// block is one GEMM on the sm_100a DMMA tile kernel (dgemm_tile.cu), and at order <= 64 a
+// base kernel works on 64 vectors per CTA staged in shared memory next to the triangle:
+// 16 x 16 diagonal blocks one thread per vector, the updates between blocks on DMMA (see
+// trxm_base_kernel).  Blocking keeps the substitution backward stable (no explicit inverse),
+// so the componentwise residual bound of DESIGN.md reading Q13 holds.
 //
 // Only the triangle op(A) references is read; with diag == 'U' the diagonal is not read.
 #include <cuda_runtime.h>
@@ -20,192 +21,232 @@ namespace {
 
 constexpr int NB = 64;  // base-case order
 
-// op(A)(r, c) of a diagonal tile stored at A (column-major, ld), trans = op is A^T
-__device__ __forceinline__ double opa(const double *A, int64_t lda, bool trans, int r, int c) {
-    return trans ? A[c + (int64_t)r * lda] : A[r + (int64_t)c * lda];
-}
 
-// One thread per vector.  The system (or product) is on vectors v of length n (n <= NB):
-//   left  side: v = a column of B (element stride 1, vectors ldb apart), matrix M = op(A)
-//   right side: v = a row of B (element stride ldb, vectors 1 apart),   matrix M = op(A)^T
-// LOWER: M is lower triangular (forward substitution / bottom-up product).
-// One launch covers the vectors of every B tile of a batch (all share the triangle).
-#ifndef XK_VPC
-#define XK_VPC 128
+// Base case (order n <= NB = 64) on the vectors of every B tile of a batch (all share the
+// triangle): left side, the vectors are the columns of B and the matrix is M = op(A); right
+// side, the vectors are the rows of B and M = op(A)^T.  A CTA takes NVB = 64 vectors (2 NVB
+// threads) and stages them in shared memory as X (one vector per padded row), next to M.  The
+// triangle is processed in diagonal blocks of BS = 16:
+//   TRSM (lower, forward): for each block kb in order, one thread per vector solves the
+//     16 x 16 diagonal block against its 16 entries (reciprocal diagonal, no inverse of the
+//     triangle), then the 4 warps update the rows below with the solved block on the FP64
+//     tensor path: X(rows > kb, :) -= M(rows > kb, kb) X(kb, :), 8 x 8 output tiles of
+//     mma.sync.m8n8k4.f64 (DMMA), 4 k-steps each.  Upper: the mirror image, blocks backward.
+//   TRMM (lower, bottom-up): for each block kb from the last, one thread per vector forms
+//     M(kb, kb) X(kb) in place (rows bottom-up), then the warps add M(kb, < kb) X(< kb, :) --
+//     blocks < kb are still unmodified.  Upper: top-down, adding M(kb, > kb) X(> kb, :).
+// Straight-line code stays small (the old one-vector-per-thread substitution over all 64
+// rows was ~3k instructions and instruction-fetch bound, profiles/r01_trsm_base_v2_ncu.txt).
+// Blocked substitution with GEMM updates is the standard backward-stable form; it is the
+// same algorithm the recursion above applies at larger orders (Q13 bounds hold).
+#ifndef XK_NVB
+#define XK_NVB 64
 #endif
-constexpr int VPC = XK_VPC;  // vectors (threads) per CTA: the triangle load is shared by all
-static_assert(VPC % 32 == 0 && (NB * NB) % VPC == 0, "VPC: whole warps, triangle split evenly");
+#ifndef XK_BS
+#define XK_BS 16
+#endif
+constexpr int BS = XK_BS;   // diagonal block of the base case
+constexpr int NVB = XK_NVB; // vectors per CTA
+constexpr int BT = 2 * NVB; // threads per CTA
+constexpr int NW = BT / 32; // warps per CTA
+constexpr int LDM = 68;   // M stride in doubles: 68 = 4 mod 16 -> conflict-free DMMA A fragments
+constexpr int LDV = 68;   // X stride per vector: conflict-free DMMA B fragments
+static_assert(NB % BS == 0 && BS % 8 == 0 && NVB % 8 == 0 && NVB <= BT, "base-case blocking");
 struct BaseBatch {
     int n;                            // tiles
-    int cta_start[kMaxBatch + 1];     // CTAs per tile: ceil(nvec / VPC)
+    int cta_start[kMaxBatch + 1];     // CTAs per tile: ceil(nvec / NVB)
     double *B[kMaxBatch];
     int64_t ldb[kMaxBatch], nvec[kMaxBatch];
+    bool al16;                        // every B and ldb 16-byte aligned: 16-byte async copies
 };
+constexpr size_t kBaseSmem = (size_t)(NB * LDM + NB + NVB * LDV) * sizeof(double);
 
-constexpr int LDM = NB + 2;  // triangle stride in shared memory (16-byte aligned rows)
+__device__ __forceinline__ void dmma884(double (&c)[2], double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c[0]), "+d"(c[1])
+                 : "d"(a), "d"(b));
+}
 
-constexpr int LDV = NB + 2;  // staged vector stride (left side): 16-byte rows, odd in 16-byte units
-constexpr size_t kBaseSmemLeft = (size_t)(NB * LDM + NB + VPC * LDV) * sizeof(double);
+// X(r0..r1, :) += sign * M(r0..r1, k0..k0+nk) X(k0..k0+nk, :) on 8 x 8 output tiles dealt to
+// the CTA's warps (sign = -1: TRSM update, +1: TRMM contribution).  A warp keeps UT tiles in
+// flight at once (independent accumulators), so the DMMA latency of one tile's k-chain is
+// hidden behind the others'.
+constexpr int UT = 4;
+__device__ __forceinline__ void block_update(const double *Ms, double *X, int r0, int r1, int k0, int nk,
+                                             double sign, int warp, int lane) {
+    const int nrt = (r1 - r0) / 8, tiles = nrt * (NVB / 8);
+    const int fr = lane >> 2, fc = lane & 3;
+    for (int t0 = warp * UT; t0 < tiles; t0 += NW * UT) {
+        int rr[UT], vv[UT];
+        double d[UT][2];
+#pragma unroll
+        for (int u = 0; u < UT; ++u) {
+            const int t = t0 + u < tiles ? t0 + u : t0;  // past the end: redo tile t0, not stored
+            rr[u] = r0 + (t % nrt) * 8;
+            vv[u] = (t / nrt) * 8;
+            d[u][0] = X[(vv[u] + 2 * fc) * LDV + rr[u] + fr];
+            d[u][1] = X[(vv[u] + 2 * fc + 1) * LDV + rr[u] + fr];
+        }
+        for (int k = 0; k < nk; k += 4) {
+#pragma unroll
+            for (int u = 0; u < UT; ++u) {
+                const double a = sign * Ms[(k0 + k + fc) * LDM + rr[u] + fr];
+                const double b = X[(vv[u] + fr) * LDV + k0 + k + fc];
+                dmma884(d[u], a, b);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < UT; ++u) {
+            if (t0 + u >= tiles) break;
+            X[(vv[u] + 2 * fc) * LDV + rr[u] + fr] = d[u][0];
+            X[(vv[u] + 2 * fc + 1) * LDV + rr[u] + fr] = d[u][1];
+        }
+    }
+}
+
+__device__ __forceinline__ void cp_async8(double *dst, const double *src, bool ok) {
+    const uint32_t d = static_cast<uint32_t>(__cvta_generic_to_shared(dst));
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(ok ? 8 : 0) : "memory");
+}
+__device__ __forceinline__ void cp_async16(double *dst, const double *src, bool ok) {
+    const uint32_t d = static_cast<uint32_t>(__cvta_generic_to_shared(dst));
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src), "r"(ok ? 16 : 0) : "memory");
+}
 
 template <bool SOLVE, bool LOWER, bool LEFT>
-__global__ void __launch_bounds__(VPC) trxm_base_kernel(const __grid_constant__ BaseBatch bb, int n,
-                                                        double alpha, const double *A, int64_t lda,
-                                                        bool mtrans, bool unit) {
-    // SOLVE: Ms[c * LDM + i] = M(i, c) (columns contiguous: column-oriented substitution);
-    // multiply: Ms[i * LDM + c] = M(i, c) (rows contiguous: row dot products).  Either way
-    // the inner loop reads two consecutive entries with one 16-byte shared load, and every
-    // thread of the warp reads the same address (broadcast).
+__global__ void __launch_bounds__(BT) trxm_base_kernel(const __grid_constant__ BaseBatch bb, int n,
+                                                       double alpha, const double *A, int64_t lda,
+                                                       bool mtrans, bool unit) {
     extern __shared__ __align__(16) double smem_base[];
-    double *Ms = smem_base;
+    double *Ms = smem_base;      // Ms[c * LDM + i] = M(i, c)
     double *rd = Ms + NB * LDM;  // 1 / M(l, l)
-    double *V = rd + NB;         // left side: the CTA's vectors, V[v * LDV + e]
+    double *X = rd + NB;         // X[v * LDV + l] = entry l of vector v
     int q = 0;
 #pragma unroll 1
     while (q + 1 < bb.n && (int)blockIdx.x >= bb.cta_start[q + 1]) ++q;
     double *B = bb.B[q];
     const int64_t ldb = bb.ldb[q], nvec = bb.nvec[q];
-    const int tid = threadIdx.x;
-    const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * VPC;
-    const int nv = (int)((nvec - v0) < VPC ? (nvec - v0) : VPC);
-    // triangle of M into shared memory, padded to NB with the identity (only the referenced
-    // part of A is read); consecutive threads read along the stored-contiguous direction,
-    // every load in flight before the first shared store (latency-bound phase)
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int64_t v0 = (int64_t)(blockIdx.x - bb.cta_start[q]) * NVB;
+    const int nv = (int)((nvec - v0) < NVB ? (nvec - v0) : NVB);
+    // Every global load is an asynchronous copy straight into shared memory (cp.async,
+    // zero-filled when predicated off), all in flight at once: the referenced triangle of M
+    // (consecutive threads along A's stored-contiguous direction; the other triangle, the
+    // unit diagonal and the padding to NB are never read from A), then the CTA's vectors.
     {
-        double t[NB * NB / VPC];
-#pragma unroll
-        for (int k = 0; k < NB * NB / VPC; ++k) {
-            const int e = tid + k * VPC, f = e % NB, s2 = e / NB;
+#pragma unroll 4
+        for (int k = 0; k < NB * NB / BT; ++k) {
+            const int e = tid + k * BT, f = e % NB, s2 = e / NB;
             const int i = mtrans ? s2 : f, c = mtrans ? f : s2;  // M(i, c); A contiguous in f
             const bool in = LOWER ? (i > c) : (i < c);
-            double v = (i == c) ? 1.0 : 0.0;
-            if (i < n && c < n && (in || (i == c && !unit))) v = opa(A, lda, mtrans, i, c);
-            t[k] = v;
+            const bool rd_a = i < n && c < n && (in || (i == c && !unit));
+            cp_async8(Ms + c * LDM + i, rd_a ? (mtrans ? A + c + (int64_t)i * lda : A + i + (int64_t)c * lda) : A, rd_a);
         }
-#pragma unroll
-        for (int k = 0; k < NB * NB / VPC; ++k) {
-            const int e = tid + k * VPC, f = e % NB, s2 = e / NB;
-            const int i = mtrans ? s2 : f, c = mtrans ? f : s2;
-            Ms[SOLVE ? c * LDM + i : i * LDM + c] = t[k];
-            if (SOLVE && i == c) rd[i] = 1.0 / t[k];
-        }
-    }
-    double x[NB];
-    if (LEFT) {
-        // vectors are columns of B (contiguous): a warp loads whole columns, 16 bytes per
-        // lane (fully coalesced), into the staging area; each thread then takes its own
-        const int w = tid >> 5, lane = tid & 31;
-        double2 u[32];  // VPC / 32 warps x 32 columns each = VPC vectors
-#pragma unroll
-        for (int k = 0; k < 32; ++k) {
-            const int v = w * 32 + k, e = 2 * lane;
-            double2 z = make_double2(0.0, 0.0);
-            if (v < nv && e < n) {
-                const double *src = B + (v0 + v) * ldb + e;
-                if (e + 1 < n) z = *reinterpret_cast<const double2 *>(src);
-                else z.x = src[0];
+        if (LEFT) {  // columns of B: a warp reads whole 512-byte columns, 16 bytes per lane
+#pragma unroll 4
+            for (int k = 0; k < NVB / NW; ++k) {
+                const int v = warp + NW * k, e = 2 * lane;
+                const bool ok = v < nv && e < n;
+                const double *src = ok ? B + (v0 + v) * ldb + e : B;
+                if (bb.al16 && (e + 1 < n || !ok)) {
+                    cp_async16(X + v * LDV + e, src, ok);
+                } else {
+                    cp_async8(X + v * LDV + e, src, ok);
+                    cp_async8(X + v * LDV + e + 1, ok && e + 1 < n ? src + 1 : B, ok && e + 1 < n);
+                }
             }
-            u[k] = z;
+        } else {     // rows of B: consecutive threads read consecutive rows of one column
+#pragma unroll 4
+            for (int k = 0; k < NB * NVB / BT; ++k) {
+                const int e = tid + k * BT, v = e % NVB, l = e / NVB;
+                const bool ok = v < nv && l < n;
+                cp_async8(X + v * LDV + l, ok ? B + (v0 + v) + (int64_t)l * ldb : B, ok);
+            }
         }
-#pragma unroll
-        for (int k = 0; k < 32; ++k) {
-            const int v = w * 32 + k;
-            *reinterpret_cast<double2 *>(V + v * LDV + 2 * lane) = u[k];
+        asm volatile("cp.async.wait_all;\n" ::: "memory");
+        __syncthreads();
+        if (tid < NB) {  // the diagonal: 1 where A's is not read (unit, padding), reciprocal
+            if (unit || tid >= n) Ms[tid * LDM + tid] = 1.0;
+            rd[tid] = 1.0 / Ms[tid * LDM + tid];
         }
         __syncthreads();
-#pragma unroll
-        for (int p = 0; p < NB / 2; ++p) {
-            const double2 z = *reinterpret_cast<const double2 *>(V + tid * LDV + 2 * p);
-            x[2 * p] = z.x;
-            x[2 * p + 1] = z.y;
-        }
-    } else {
-        // vectors are rows of B: consecutive threads read consecutive addresses
-        const bool active = tid < nv;
-        const double *p = B + (v0 + tid);
-#pragma unroll
-        for (int i = 0; i < NB; ++i, p += ldb) x[i] = (active && i < n) ? *p : 0.0;
     }
-    __syncthreads();
-    if (SOLVE) {
+    constexpr int NBLK = NB / BS;
+#pragma unroll 1
+    for (int step = 0; step < NBLK; ++step) {
+        // block order: TRSM lower / TRMM upper forward, the others backward
+        const int kb = (SOLVE == LOWER) ? step : NBLK - 1 - step;
+        const int o = kb * BS;
+        if (tid < NVB) {  // one thread per vector: the diagonal block
+            double *xv = X + tid * LDV + o;
+            double x[BS];
 #pragma unroll
-        for (int i = 0; i < NB; ++i) x[i] *= alpha;
-        if (LOWER) {  // column-oriented forward substitution: x_i -= M_il x_l, l ascending
+            for (int p = 0; p < BS / 2; ++p) {
+                const double2 z = *reinterpret_cast<const double2 *>(xv + 2 * p);
+                x[2 * p] = z.x;
+                x[2 * p + 1] = z.y;
+            }
+            if (SOLVE && LOWER) {         // forward, column-oriented
 #pragma unroll
-            for (int l = 0; l < NB; ++l) {
-                if (!unit) x[l] *= rd[l];
-                const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
+                for (int l = 0; l < BS; ++l) {
+                    if (!unit) x[l] *= rd[o + l];
 #pragma unroll
-                for (int p = (l + 1) / 2; p < NB / 2; ++p) {
-                    const double2 m2 = col[p];
-                    if (2 * p > l) x[2 * p] -= m2.x * x[l];
-                    x[2 * p + 1] -= m2.y * x[l];
+                    for (int i = l + 1; i < BS; ++i) x[i] -= Ms[(o + l) * LDM + o + i] * x[l];
+                }
+            } else if (SOLVE) {           // backward
+#pragma unroll
+                for (int l = BS - 1; l >= 0; --l) {
+                    if (!unit) x[l] *= rd[o + l];
+#pragma unroll
+                    for (int i = 0; i < l; ++i) x[i] -= Ms[(o + l) * LDM + o + i] * x[l];
+                }
+            } else if (LOWER) {           // bottom-up: row i reads x_0..x_i, still unmodified
+#pragma unroll
+                for (int i = BS - 1; i >= 0; --i) {
+                    double s = 0.0;
+#pragma unroll
+                    for (int l = 0; l <= i; ++l) s += Ms[(o + l) * LDM + o + i] * x[l];
+                    x[i] = s;
+                }
+            } else {                      // top-down: row i reads x_i..x_BS-1
+#pragma unroll
+                for (int i = 0; i < BS; ++i) {
+                    double s = 0.0;
+#pragma unroll
+                    for (int l = i; l < BS; ++l) s += Ms[(o + l) * LDM + o + i] * x[l];
+                    x[i] = s;
                 }
             }
-        } else {      // back substitution, l descending
 #pragma unroll
-            for (int l = NB - 1; l >= 0; --l) {
-                if (!unit) x[l] *= rd[l];
-                const double2 *col = reinterpret_cast<const double2 *>(Ms + l * LDM);
-#pragma unroll
-                for (int p = 0; 2 * p < l; ++p) {
-                    const double2 m2 = col[p];
-                    x[2 * p] -= m2.x * x[l];
-                    if (2 * p + 1 < l) x[2 * p + 1] -= m2.y * x[l];
-                }
-            }
+            for (int p = 0; p < BS / 2; ++p)
+                *reinterpret_cast<double2 *>(xv + 2 * p) = make_double2(x[2 * p], x[2 * p + 1]);
         }
-    } else {
-        if (LOWER) {  // bottom-up: row i only reads x_0..x_i, still unmodified
-#pragma unroll
-            for (int i = NB - 1; i >= 0; --i) {
-                const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
-                double s = 0.0;
-#pragma unroll
-                for (int p = 0; 2 * p <= i; ++p) {
-                    const double2 m2 = row[p];
-                    s += m2.x * x[2 * p];
-                    if (2 * p + 1 <= i) s += m2.y * x[2 * p + 1];
-                }
-                x[i] = alpha * s;
-            }
-        } else {      // top-down: row i only reads x_i..x_NB-1, still unmodified
-#pragma unroll
-            for (int i = 0; i < NB; ++i) {
-                const double2 *row = reinterpret_cast<const double2 *>(Ms + i * LDM);
-                double s = 0.0;
-#pragma unroll
-                for (int p = i / 2; p < NB / 2; ++p) {
-                    const double2 m2 = row[p];
-                    if (2 * p >= i) s += m2.x * x[2 * p];
-                    s += m2.y * x[2 * p + 1];
-                }
-                x[i] = alpha * s;
-            }
-        }
-    }
-    if (LEFT) {
-        // back through the staging area so that every warp stores whole columns
-#pragma unroll
-        for (int p = 0; p < NB / 2; ++p)
-            *reinterpret_cast<double2 *>(V + tid * LDV + 2 * p) = make_double2(x[2 * p], x[2 * p + 1]);
         __syncthreads();
-        const int w = tid >> 5, lane = tid & 31;
+        if (SOLVE && LOWER) block_update(Ms, X, o + BS, NB, o, BS, -1.0, warp, lane);
+        else if (SOLVE) block_update(Ms, X, 0, o, o, BS, -1.0, warp, lane);
+        else if (LOWER) block_update(Ms, X, o, o + BS, 0, o, 1.0, warp, lane);
+        else block_update(Ms, X, o, o + BS, o + BS, NB - o - BS, 1.0, warp, lane);
+        __syncthreads();
+    }
+    // X back to B, times alpha (TRSM: op(A)^-1 (alpha B) = alpha op(A)^-1 B)
+    const double so = alpha;
+    if (LEFT) {
 #pragma unroll
-        for (int k = 0; k < 32; ++k) {
-            const int v = w * 32 + k, e = 2 * lane;
+        for (int k = 0; k < NVB / NW; ++k) {
+            const int v = warp + NW * k, e = 2 * lane;
             if (v < nv && e < n) {
-                const double2 z = *reinterpret_cast<const double2 *>(V + v * LDV + e);
+                const double2 z = *reinterpret_cast<const double2 *>(X + v * LDV + e);
                 double *dst = B + (v0 + v) * ldb + e;
-                if (e + 1 < n) *reinterpret_cast<double2 *>(dst) = z;
-                else dst[0] = z.x;
+                if (e + 1 < n) *reinterpret_cast<double2 *>(dst) = make_double2(so * z.x, so * z.y);
+                else dst[0] = so * z.x;
             }
         }
-    } else if (tid < nv) {
-        double *p = B + (v0 + tid);
-        asm volatile("mov.b64 %0, %0;" : "+l"(p));  // opaque: no CSE with the load addresses
+    } else {
 #pragma unroll
-        for (int i = 0; i < NB; ++i, p += ldb)
-            if (i < n) *p = x[i];
+        for (int k = 0; k < NB * NVB / BT; ++k) {
+            const int e = tid + k * BT, v = e % NVB, l = e / NVB;
+            if (v < nv && l < n) B[(v0 + v) + (int64_t)l * ldb] = so * X[v * LDV + l];
+        }
     }
 }
 
@@ -232,16 +273,15 @@ template <bool SOLVE, bool LOWER, bool LEFT>
 cudaError_t base_launch(const BaseBatch &bb, unsigned grid, int n, double alpha, const double *A,
                         int64_t lda, bool mtrans, bool unit, cudaStream_t st) {
     auto kern = trxm_base_kernel<SOLVE, LOWER, LEFT>;
-    const size_t smem = LEFT ? kBaseSmemLeft : (size_t)(NB * LDM + NB) * sizeof(double);
     static unsigned attr_set = 0;  // per instantiation, one bit per device
     int dev = 0;
     cudaGetDevice(&dev);
     if (!(attr_set & (1u << dev))) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBaseSmemLeft);
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBaseSmem);
         if (e != cudaSuccess) return e;
         attr_set |= 1u << dev;
     }
-    kern<<<grid, VPC, smem, st>>>(bb, n, alpha, A, lda, mtrans, unit);
+    kern<<<grid, BT, kBaseSmem, st>>>(bb, n, alpha, A, lda, mtrans, unit);
     return cudaGetLastError();
 }
 
@@ -249,13 +289,15 @@ cudaError_t base(const TriOp &o, int64_t n, const Tiles &T, double alpha, const 
                  cudaStream_t st) {
     BaseBatch bb;
     bb.n = T.n;
+    bb.al16 = true;
     int total = 0;
     for (int q = 0; q < T.n; ++q) {
         bb.cta_start[q] = total;
         bb.B[q] = T.B[q];
         bb.ldb[q] = T.ldb[q];
         bb.nvec[q] = T.other[q];
-        total += (int)((T.other[q] + VPC - 1) / VPC);
+        bb.al16 = bb.al16 && ((uintptr_t)T.B[q] % 16 == 0) && (T.ldb[q] % 2 == 0);
+        total += (int)((T.other[q] + NVB - 1) / NVB);
     }
     bb.cta_start[T.n] = total;
     if (total == 0) return cudaSuccess;

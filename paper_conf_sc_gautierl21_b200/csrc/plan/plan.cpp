@@ -76,6 +76,8 @@ int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t
                 }
                 for (auto it = keymap_.begin(); it != keymap_.end();)
                     if (entries_[it->second].mat == (int)i) it = keymap_.erase(it); else ++it;
+                M.grid.clear();
+                M.gr = M.gc = 0;
                 M.rows = rows;
                 M.cols = cols;
                 return (int)i;
@@ -105,6 +107,8 @@ int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t
             }
             for (auto it = keymap_.begin(); it != keymap_.end();)
                 if (entries_[it->second].mat == (int)i) it = keymap_.erase(it); else ++it;
+            M.grid.clear();
+            M.gr = M.gc = 0;
             M.ld = -1;  // forget
         }
     }
@@ -118,9 +122,25 @@ int Planner::find_or_add_matrix(uint64_t base, int64_t ld, int64_t rows, int64_t
 }
 
 int Planner::key_of(int mat, int64_t bi, int64_t bj) {
+    Matrix &Mx = mats_[mat];
+    const int64_t tr = cdiv(Mx.rows, flags_.T), tc = cdiv(Mx.cols, flags_.T);
+    if (Mx.gr != tr || Mx.gc != tc) {  // (re)build the dense cache from the directory
+        Mx.grid.assign((size_t)(tr * tc), -1);
+        Mx.gr = tr;
+        Mx.gc = tc;
+        for (const auto &kv : keymap_) {
+            const Entry &e = entries_[kv.second];
+            if (e.mat == mat && e.bi < tr && e.bj < tc) Mx.grid[(size_t)(e.bi + e.bj * tr)] = kv.second;
+        }
+    }
+    const bool in_grid = bi < tr && bj < tc;
+    if (in_grid && Mx.grid[(size_t)(bi + bj * tr)] >= 0) return Mx.grid[(size_t)(bi + bj * tr)];
     const uint64_t k = tile_key(mat, bi, bj);
     auto it = keymap_.find(k);
-    if (it != keymap_.end()) return it->second;
+    if (it != keymap_.end()) {
+        if (in_grid) Mx.grid[(size_t)(bi + bj * tr)] = it->second;
+        return it->second;
+    }
     Entry e;
     e.mat = mat;
     e.bi = bi;
@@ -135,6 +155,7 @@ int Planner::key_of(int mat, int64_t bi, int64_t bj) {
     entries_.push_back(e);
     int id = (int)entries_.size() - 1;
     keymap_[k] = id;
+    if (in_grid) mats_[mat].grid[(size_t)(bi + bj * tr)] = id;
     return id;
 }
 
@@ -454,14 +475,26 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
     for (auto &kv : last) tasks[kv.second].last_writer = true;
     out.reserve(out.size() + tasks.size() * 2);
     std::vector<std::vector<int>> lists(G);
-    for (size_t q = 0; q < tasks.size(); ++q) lists[tasks[q].gpu].push_back((int)q);
-    for (int d = 0; d < G; ++d) {
-        std::stable_sort(lists[d].begin(), lists[d].end(), [&](int a, int b) {
-            const Task &x = tasks[a], &y = tasks[b];
-            for (int q = 0; q < 5; ++q)
-                if (x.skey[q] != y.skey[q]) return x.skey[q] < y.skey[q];
-            return false;
-        });
+    {
+        // per-GPU order by the generator's sort key (ties: generation order), sorted on a
+        // compact copy of the keys rather than through the large Task records
+        struct SK { int64_t k[5]; int idx; };
+        std::vector<std::vector<SK>> keys(G);
+        for (size_t q = 0; q < tasks.size(); ++q) {
+            SK s;
+            std::copy(tasks[q].skey, tasks[q].skey + 5, s.k);
+            s.idx = (int)q;
+            keys[tasks[q].gpu].push_back(s);
+        }
+        for (int d = 0; d < G; ++d) {
+            std::sort(keys[d].begin(), keys[d].end(), [](const SK &x, const SK &y) {
+                for (int q = 0; q < 5; ++q)
+                    if (x.k[q] != y.k[q]) return x.k[q] < y.k[q];
+                return x.idx < y.idx;
+            });
+            lists[d].reserve(keys[d].size());
+            for (const SK &s : keys[d]) lists[d].push_back(s.idx);
+        }
     }
     std::vector<size_t> pos(G, 0);
     auto ready = [&](const Task &t) {
@@ -600,6 +633,8 @@ static char up(char c) { return (c >= 'a' && c <= 'z') ? (char)(c - 32) : c; }
 int Planner::add_shadow(int mc) {
     Matrix S = mats_[mc];
     S.shadow = true;
+    S.grid.clear();  // its own tiles (never C's cached ids)
+    S.gr = S.gc = 0;
     mats_.push_back(S);
     return (int)mats_.size() - 1;
 }
@@ -623,6 +658,8 @@ void Planner::drop_shadow(int ms) {
             ++it;
         }
     }
+    mats_[ms].grid.clear();
+    mats_[ms].gr = mats_[ms].gc = 0;
     mats_[ms].ld = -1;
 }
 

@@ -43,6 +43,10 @@ struct Matrix {
     int64_t rows = 0, cols = 0;  // stored extent covered by the tiles known so far
     bool shadow = false;         // per-call read-only view of C's input values (beta deferral)
     bool host_once = false;      // shadow read from the host at most once (R15: TRMM's B)
+    // dense (bi, bj) -> directory id cache of keymap_ for this matrix (-1 = not yet looked
+    // up); rebuilt when the tile grid grows, cleared when the matrix's entries are forgotten
+    std::vector<int> grid;
+    int64_t gr = 0, gc = 0;
 };
 
 struct NodeCopy {

@@ -64,7 +64,7 @@ def build_xk(force=False, verbose=False):
     for s in cu:
         o = os.path.join(objdir, os.path.basename(s) + ".o")
         objs.append(o)
-        cmd = [NVCC] + ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
+        cmd = [NVCC] + ARCH + os.environ.get("XK_NVCC_FLAGS", "").split() + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
                                "-Xptxas", "-v" if verbose else "-O3", "-c", s, "-o", o] + inc
         procs.append((cmd, subprocess.Popen(cmd, cwd=ROOT, stdout=subprocess.PIPE,
                                             stderr=subprocess.STDOUT, text=True)))
