@@ -236,13 +236,16 @@ def make_inputs(N):
     return A, B, C
 
 
-def traffic_from_profiles(T):
+def traffic_from_profiles(T, tasks_per_launch):
+    """DRAM bytes per launch for the roofline: the committed ncu capture's bytes per tile task
+    (one full capture of a grouped launch at this tile size) times the average tasks per
+    launch of the timed pass -- per launch, like `achieved`."""
     p = os.path.join(ROOT, "profiles", "dgemm_tile_ncu.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        if int(d.get("tile", 0)) == T:
-            return d.get("dram_bytes_per_launch")
+        if int(d.get("tile", 0)) == T and d.get("tasks_per_launch"):
+            return d["dram_bytes_per_launch"] / d["tasks_per_launch"] * tasks_per_launch
     except (OSError, ValueError):
         pass
     return None
@@ -567,7 +570,11 @@ def assemble_line(args, G, ws, N, T, host, t_roof, terms, bw_src, dod, avg_ms, f
     mode = "rank mode: one process per GPU" if ws > 1 else "one process"
     grid = "x".join(map(str, _grid(G)))
     roof = {"bound": "tensor", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
-            "frac": (achieved / FP64_PEAK_TFLOPS) if achieved else None, "traffic": traffic_from_profiles(T),
+            "frac": (achieved / FP64_PEAK_TFLOPS) if achieved else None,
+            "traffic": traffic_from_profiles(T, flops_per_launch / (2.0 * T ** 3)),
+            "traffic_note": "ncu dram__bytes_read+write of one grouped launch (profiles/dgemm_tile_ncu.json) per tile "
+                            "task x the average tasks per timed launch; algorithmic %.3g bytes per launch (A, B, C "
+                            "read + C write per task)" % (4 * 8.0 * T * T * flops_per_launch / (2.0 * T ** 3)),
             "kernel": "dgemm_tma_kernel (grouped launch; TMA + mbarrier pipeline; FP64 DMMA.8x8x4 via mma.sync.m8n8k4.f64)",
             "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 x 1965 MHz (no FP64 entry in "
                            "MEASURED_PEAKS.json); DMMA microbenchmark on this pool measured 37.07",
