@@ -489,6 +489,7 @@ int Runtime::record(cudaStream_t s, int g, Ev *out) {
     XK_CK(cudaEventRecord(e, s));
     out->e = e;
     out->s = s;
+    out->c = ++rec_count_[s];
     return XK_OK;
 }
 
@@ -499,6 +500,14 @@ int Runtime::wait_on(cudaStream_t s, const Ev &ev) {
         return XK_OK;
     }
     if (!ev.e || ev.s == s) return XK_OK;  // same stream: already ordered
+    if (ev.c) {  // already waited for this event or a later one of its stream: implied
+        uint64_t &w = waited_[std::make_pair(s, ev.s)];
+        if (ev.c <= w) {
+            ++waits_skipped_;
+            return XK_OK;
+        }
+        w = ev.c;
+    }
     XK_CK(cudaStreamWaitEvent(s, ev.e, 0));
     return XK_OK;
 }

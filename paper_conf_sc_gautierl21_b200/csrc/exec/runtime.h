@@ -26,6 +26,7 @@ constexpr int kMaxKStreams = 8;
 struct Ev {
     cudaEvent_t e = nullptr;
     cudaStream_t s = nullptr;  // stream it was recorded on
+    uint64_t c = 0;            // ordinal of the record on that stream (1, 2, ...)
     int64_t rseq = -1;         // rank mode: plan record executed by another process (flag wait)
     static Ev remote(int64_t seq) { Ev v; v.rseq = seq; return v; }
 };
@@ -151,6 +152,17 @@ private:
     std::vector<Device> devs_;
     std::unordered_map<int64_t, Buffer> bufs_;  // key * XK_MAX_GPUS + g
     std::unordered_map<int64_t, Ev> seq_ev_;    // plan seq -> completion event (this epoch)
+    // event-wait deduplication: events recorded per stream, and per (waiting stream, recorded
+    // stream) the latest ordinal already waited for -- a stream's events complete in order, so
+    // waiting for a later one covers every earlier one
+    std::unordered_map<cudaStream_t, uint64_t> rec_count_;
+    struct StreamPairHash {
+        size_t operator()(const std::pair<cudaStream_t, cudaStream_t> &p) const {
+            return std::hash<const void *>()(p.first) * 31u ^ std::hash<const void *>()(p.second);
+        }
+    };
+    std::unordered_map<std::pair<cudaStream_t, cudaStream_t>, uint64_t, StreamPairHash> waited_;
+    int64_t waits_skipped_ = 0;
     std::vector<std::vector<cudaEvent_t>> ev_pool_, ev_used_;  // per logical GPU
     std::vector<Ev> pending_d2h_;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ktimers_;

@@ -32,7 +32,10 @@ constexpr int BK = 16;
 #define XK_CPF 0  // extra k-blocks of lead for the epilogue's C prefetch (-1 = off)
 #endif
 constexpr int BM = 64, BN = 128;   // CTA tile
-constexpr int WM = 32, WN = 32;    // warp tile
+#ifndef XK_WN
+#define XK_WN 32
+#endif
+constexpr int WM = 32, WN = XK_WN;  // warp tile (32 x 32: 8 warps; 32 x 64: 4 warps)
 constexpr int NWM = BM / WM, NWN = BN / WN, NWARPS = NWM * NWN;
 constexpr int NTHREADS = NWARPS * 32;
 constexpr int STAGES = 4;
@@ -188,18 +191,21 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
             // the epilogue's C (and deferred-beta C2) reads are cold DRAM reads: pull this
             // warp's 32 x 32 block into L2 while the last k-blocks still run (one column of
             // 256 bytes per lane)
-            const int64_t col = n0 + wn + lane;
             const int64_t row = m0 + wm;
-            if (col < t.N && row < t.M) {
-                if (t.beta != 0.0) {
-                    const double *pc = t.C + row + col * t.ldc;
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(pc));
-                    if (row + 16 < t.M) asm volatile("prefetch.global.L2 [%0];" ::"l"(pc + 16));
-                }
-                if (t.beta2 != 0.0) {
-                    const double *p2 = t.C2 + row + col * t.ldc2;
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(p2));
-                    if (row + 16 < t.M) asm volatile("prefetch.global.L2 [%0];" ::"l"(p2 + 16));
+#pragma unroll
+            for (int cg = 0; cg < WN / 32; ++cg) {
+                const int64_t col = n0 + wn + cg * 32 + lane;
+                if (col < t.N && row < t.M) {
+                    if (t.beta != 0.0) {
+                        const double *pc = t.C + row + col * t.ldc;
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(pc));
+                        if (row + 16 < t.M) asm volatile("prefetch.global.L2 [%0];" ::"l"(pc + 16));
+                    }
+                    if (t.beta2 != 0.0) {
+                        const double *p2 = t.C2 + row + col * t.ldc2;
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(p2));
+                        if (row + 16 < t.M) asm volatile("prefetch.global.L2 [%0];" ::"l"(p2 + 16));
+                    }
                 }
             }
         }
