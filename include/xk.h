@@ -199,6 +199,17 @@ int xk_sync(void);
 int xk_memory_invalidate(int64_t m, int64_t n, const double *A, int64_t lda);
 /* Load the tiles of a host view onto their owner GPUs now (data-on-device runs). */
 int xk_memory_prefetch_async(int64_t m, int64_t n, const double *A, int64_t lda);
+/* The paper's xkblas_distribute_2Dblock_cyclic_async (SecIV-C, "data on device"):
+ * distribute the tiles of a host view over a P x Q grid of GPUs in 2D block-cyclic blocks
+ * of mb x nb tiles (ScaLAPACK layout; the paper's runs use the (4,2) grid and (1,1) blocks):
+ * tile (bi, bj) goes to GPU ((bi / mb) mod P) * Q + ((bj / nb) mod Q).  Asynchronous; the
+ * tiles stay in the cache as valid copies, so later calls read them from the GPUs (a tile
+ * whose task runs on another GPU is forwarded over the peer links, never re-read from the
+ * host).  Tiles are the library's T x T tiles of the view anchored at A (as every call).
+ * Errors: -1 m < 0, -2 n < 0, -4 lda < max(1, m), -5 P < 1, -6 Q < 1 or P*Q > ngpus,
+ * -7 mb < 1, -8 nb < 1; XK_ERR_* as the BLAS calls. */
+int xk_distribute_2dbc_async(int64_t m, int64_t n, const double *A, int64_t lda, int P, int Q,
+                             int64_t mb, int64_t nb);
 
 /* ------------------------------------------------------------------ observability */
 typedef struct xk_stats {
@@ -291,6 +302,7 @@ int xk_probe_host_links(int64_t bytes_per_gpu);
 #define XK_ROUTINE_SYNC 101
 #define XK_ROUTINE_INVALIDATE 102
 #define XK_ROUTINE_PREFETCH 103
+#define XK_ROUTINE_DISTRIBUTE 104 /* view (m, n, C, ldc); grid_p x grid_q GPUs, blocks mb x nb tiles */
 
 typedef struct xk_flags {
     int topo, optimistic, window;
@@ -320,6 +332,8 @@ typedef struct xk_call {
     double alpha, beta;
     uint64_t A, lda, B, ldb, C, ldc;
     int sync; /* 1 = synchronous routine: D2H of the output after its last writer */
+    int grid_p, grid_q; /* XK_ROUTINE_DISTRIBUTE: GPU grid (P*Q <= G) */
+    int64_t mb, nb;     /* XK_ROUTINE_DISTRIBUTE: block-cyclic block size in tiles */
 } xk_call_t;
 
 typedef struct xk_plan_rec {

@@ -18,7 +18,7 @@ from ._abi import (HOST, REC_D2H, REC_FIELDS, REC_H2D, REC_P2P, REC_TASK, ROUTIN
 
 __all__ = ["init", "finalize", "register", "unregister", "dgemm", "dgemm_async",
            "memory_coherent_sync", "memory_coherent_async", "sync", "memory_invalidate",
-           "memory_prefetch_async", "get_stats", "reset_stats", "set_kernel_timing",
+           "memory_prefetch_async", "distribute_2dbc_async", "probe_host_links", "get_stats", "reset_stats", "set_kernel_timing",
            "get_topology", "PlanSession", "plan_dump", "dgemm_tile_device", "XKError", "lib"]
 
 TOPO_NAMES = {"ranked": TOPO_RANKED, "unranked": TOPO_UNRANKED, "home": TOPO_HOME}
@@ -200,6 +200,11 @@ def memory_prefetch_async(m, n, A, lda):
     return _check(lib().xk_memory_prefetch_async(m, n, _p(A), lda))
 
 
+def distribute_2dbc_async(m, n, A, lda, P, Q, mb=1, nb=1):
+    """xk_distribute_2dbc_async (the paper's xkblas_distribute_2Dblock_cyclic_async)."""
+    return _check(lib().xk_distribute_2dbc_async(m, n, _p(A), lda, P, Q, mb, nb))
+
+
 # ---------------------------------------------------------------------------- observability
 def get_stats():
     st = _abi.Stats()
@@ -271,8 +276,11 @@ def _flags(topo="ranked", optimistic=True, window=2, grid=(0, 0), tile=2048, mem
 
 
 def make_call(routine=ROUTINE_DGEMM, transA="N", transB="N", m=0, n=0, k=0, alpha=1.0, beta=0.0,
-              A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False, uplo="L", side="L", diag="N"):
+              A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False, uplo="L", side="L", diag="N",
+              grid=(0, 0), mb=0, nb=0):
     c = _abi.Call()
+    c.grid_p, c.grid_q = grid
+    c.mb, c.nb = mb, nb
     c.routine = routine
     c.transA, c.transB = _c(transA), _c(transB)
     c.uplo, c.side, c.diag = _c(uplo), _c(side), _c(diag)

@@ -24,6 +24,7 @@ SRC_NONE, SRC_VALID, SRC_INFLIGHT, SRC_HOST = 0, 1, 2, 3
 ROUTINE_DGEMM, ROUTINE_DSYRK, ROUTINE_DSYR2K, ROUTINE_DSYMM, ROUTINE_DTRMM, ROUTINE_DTRSM = 0, 1, 2, 3, 4, 5
 OP_GEMM, OP_SCALE, OP_GEMM_TRI, OP_SYMM_DIAG, OP_TRMM_DIAG, OP_TRSM_DIAG = 0, 1, 2, 3, 4, 5
 ROUTINE_COHERENT, ROUTINE_SYNC, ROUTINE_INVALIDATE, ROUTINE_PREFETCH = 100, 101, 102, 103
+ROUTINE_DISTRIBUTE = 104
 
 i64 = ctypes.c_int64
 u64 = ctypes.c_uint64
@@ -68,7 +69,8 @@ class Call(ctypes.Structure):
     _fields_ = [("routine", c_int), ("transA", c_char), ("transB", c_char), ("uplo", c_char),
                 ("side", c_char), ("diag", c_char), ("m", i64), ("n", i64),
                 ("k", i64), ("alpha", c_double), ("beta", c_double), ("A", u64), ("lda", u64),
-                ("B", u64), ("ldb", u64), ("C", u64), ("ldc", u64), ("sync", c_int)]
+                ("B", u64), ("ldb", u64), ("C", u64), ("ldc", u64), ("sync", c_int),
+                ("grid_p", c_int), ("grid_q", c_int), ("mb", i64), ("nb", i64)]
 
 
 class PlanRec(ctypes.Structure):
@@ -117,6 +119,7 @@ _SIGS = [
     ("xk_sync", c_int, []),
     ("xk_memory_invalidate", c_int, [i64, i64, vp, i64]),
     ("xk_memory_prefetch_async", c_int, [i64, i64, vp, i64]),
+    ("xk_distribute_2dbc_async", c_int, [i64, i64, vp, i64, c_int, c_int, i64, i64]),
     ("xk_get_stats", c_int, [ctypes.POINTER(Stats)]),
     ("xk_reset_stats", c_int, []),
     ("xk_set_kernel_timing", c_int, [c_int]),

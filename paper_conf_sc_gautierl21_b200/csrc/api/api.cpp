@@ -341,6 +341,30 @@ int xk_memory_coherent_async(int64_t m, int64_t n, double *A, int64_t lda) {
 int xk_memory_prefetch_async(int64_t m, int64_t n, const double *A, int64_t lda) {
     return view_call(XK_ROUTINE_PREFETCH, m, n, A, lda, false);
 }
+int xk_distribute_2dbc_async(int64_t m, int64_t n, const double *A, int64_t lda, int P, int Q,
+                             int64_t mb, int64_t nb) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    if (lda < imax(1, m)) return -4;
+    if (P < 1) return -5;
+    xk::Runtime *rt = runtime();
+    if (Q < 1 || (rt && (int64_t)P * Q > rt->topo.G)) return -6;
+    if (mb < 1) return -7;
+    if (nb < 1) return -8;
+    if (!rt) return need_init();
+    if (m == 0 || n == 0) return XK_OK;
+    xk_call_t c{};
+    c.routine = XK_ROUTINE_DISTRIBUTE;
+    c.m = m;
+    c.n = n;
+    c.C = (uint64_t)(uintptr_t)A;
+    c.ldc = (uint64_t)lda;
+    c.grid_p = P;
+    c.grid_q = Q;
+    c.mb = mb;
+    c.nb = nb;
+    return rt->run(c, false);
+}
 int xk_sync(void) {
     xk::Runtime *rt = runtime();
     if (!rt) return need_init();

@@ -1255,7 +1255,10 @@ int Planner::plan_coherent(const xk_call_t &c, std::vector<Rec> &out, std::strin
             for (int64_t bi = 0; bi < cdiv(c.m, T); ++bi) {
                 int key = key_of(mat, bi, bj);
                 Entry &e = entries_[key];
+                // prefetch: the owner-computes map; distribute: the caller's block-cyclic grid
                 int d = owner(bi, bj);
+                if (c.routine == XK_ROUTINE_DISTRIBUTE)
+                    d = (int)(((bi / c.mb) % c.grid_p) * c.grid_q + ((bj / c.nb) % c.grid_q));
                 if (e.gpu[d].present && e.gpu[d].ver == e.ver) continue;
                 if (!emit_copy(key, e.ver, d, 0, 2, out)) {
                     err = "prefetch: no valid copy of a tile";
@@ -1454,6 +1457,12 @@ int Planner::plan_impl(const xk_call_t &c, std::vector<Rec> &out, std::string &e
         invalidate(c.C, c.m, c.n, (int64_t)c.ldc);
         return XK_OK;
     case XK_ROUTINE_PREFETCH:
+        return plan_coherent(c, out, err, true);
+    case XK_ROUTINE_DISTRIBUTE:
+        if (c.grid_p < 1 || c.grid_q < 1 || (int64_t)c.grid_p * c.grid_q > topo_.G || c.mb < 1 || c.nb < 1) {
+            err = "distribute: need 1 <= P*Q <= ngpus and block sizes >= 1";
+            return XK_ERR_CONFIG;
+        }
         return plan_coherent(c, out, err, true);
     default:
         err = "unknown routine";

@@ -21,7 +21,7 @@ S_NONE, S_VALID, S_INFLIGHT, S_HOST = 0, 1, 2, 3
 RANKED, UNRANKED, HOME = 0, 1, 2
 HOSTID = -1
 DGEMM, DSYRK, DSYR2K, DSYMM, DTRMM, DTRSM = 0, 1, 2, 3, 4, 5
-COHERENT, SYNC, INVALIDATE, PREFETCH = 100, 101, 102, 103
+COHERENT, SYNC, INVALIDATE, PREFETCH, DISTRIBUTE = 100, 101, 102, 103, 104
 OP_GEMM, OP_SCALE, OP_GEMM_TRI, OP_SYMM_DIAG, OP_TRMM_DIAG, OP_TRSM_DIAG = 0, 1, 2, 3, 4, 5
 
 
@@ -224,7 +224,8 @@ class Model:
 
     # ------------------------------------------------------------------ calls
     def call(self, routine=DGEMM, transA="N", transB="N", m=0, n=0, k=0, alpha=1.0, beta=0.0,
-             A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False, uplo="L", side="L", diag="N"):
+             A=0, lda=1, B=0, ldb=1, C=0, ldc=1, sync=False, uplo="L", side="L", diag="N",
+             grid=(0, 0), mb=0, nb=0):
         out = []
         ta, tb = transA.upper() in "TC", transB.upper() in "TC"
         lower, left = uplo.upper() == "L", side.upper() == "L"
@@ -281,6 +282,9 @@ class Model:
             self.invalidate(C, (m, n), ldc)
         elif routine == PREFETCH:
             self.prefetch(C, m, n, ldc, out)
+        elif routine == DISTRIBUTE:
+            P, Q = grid
+            self.prefetch(C, m, n, ldc, out, owner=lambda bi, bj: ((bi // mb) % P) * Q + (bj // nb) % Q)
         return out
 
     # ---- task generators: program order, symbolic versions (readings in DESIGN.md)
@@ -720,7 +724,7 @@ class Model:
         for t, src, sub in wb:
             self.copy_out(t, src, sub, t.gpus[src].t_done, t.gpus[src].producer, out)
 
-    def prefetch(self, base, m, n, ld, out):
+    def prefetch(self, base, m, n, ld, out, owner=None):
         if m <= 0 or n <= 0:
             return
         self.matrix(base, ld, m, n)
@@ -728,7 +732,7 @@ class Model:
         for bj in range(ceil_div(n, T)):
             for bi in range(ceil_div(m, T)):
                 t = self.tile(base, ld, bi, bj)
-                d = self.owner(bi, bj)
+                d = (owner or self.owner)(bi, bj)
                 c = t.gpus.get(d)
                 if c is not None and c.ver == t.ver:
                     continue

@@ -58,6 +58,14 @@ def test_argument_errors_match_oracle_codes():
     for f, of in ((xk.dtrmm, oracle.dtrmm), (xk.dtrsm, oracle.dtrsm)):
         assert f("L", "L", "N", "X", 2, 2, 1.0, A, 4, A, 4) == of("L", "L", "N", "X", 2, 2, 1.0, A, A) == -4
         assert f("L", "L", "N", "N", 4, 2, 1.0, A, 4, A, 3) == -11
+    # xk_distribute_2dbc_async: argument codes checked before the library state
+    assert xk.lib().xk_distribute_2dbc_async(-1, 2, None, 4, 1, 1, 1, 1) == -1
+    assert xk.lib().xk_distribute_2dbc_async(2, -1, None, 4, 1, 1, 1, 1) == -2
+    assert xk.lib().xk_distribute_2dbc_async(5, 2, None, 4, 1, 1, 1, 1) == -4
+    assert xk.lib().xk_distribute_2dbc_async(4, 2, None, 4, 0, 1, 1, 1) == -5
+    assert xk.lib().xk_distribute_2dbc_async(4, 2, None, 4, 1, 0, 1, 1) == -6
+    assert xk.lib().xk_distribute_2dbc_async(4, 2, None, 4, 1, 1, 0, 1) == -7
+    assert xk.lib().xk_distribute_2dbc_async(4, 2, None, 4, 1, 1, 1, 0) == -8
 
 
 def test_product_never_imports_the_oracle():

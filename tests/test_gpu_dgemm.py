@@ -388,3 +388,39 @@ def test_async_then_sync_then_coherent(G):
     refF = np.zeros((N, N), order="F")
     oracle.dgemm("N", "N", N, N, N, 1.0, X, C2, 0.0, refF)
     check_bound("N", "N", N, N, N, 1.0, X, C2, 0.0, refF, F2, refF)
+
+
+@pytest.mark.parametrize("grid", [(2, 4), (4, 2)])
+def test_distribute_2dbc_then_dgemm(grid):
+    """Data on device the paper's way (xkblas_distribute_2Dblock_cyclic_async):
+    A, B, C distributed over 8 logical GPUs on a (P, Q) grid with (1, 1) blocks, then an async
+    DGEMM: no byte crosses PCIe during the call (H2D = 0), every tile one H2D in the
+    distribution; exact integers, bitwise vs the oracle after coherence."""
+    N, T = 768, 128
+    A, B, C0 = inputs.integers(1, N, N), inputs.integers(2, N, N), inputs.integers(3, N, N)
+    C = C0.copy(order="F")
+    ref = C0.copy(order="F")
+    oracle.dgemm("N", "N", N, N, N, 2.0, A, B, -1.0, ref)
+    logical(8, tile=T)
+    try:
+        xk.reset_stats()
+        for X in (A, B, C):
+            assert xk.distribute_2dbc_async(N, N, X, N, *grid) == 0
+        xk.sync()
+        st = xk.get_stats()
+        assert sum(st["h2d_bytes"]) == 3 * 8 * N * N
+        P, Q = grid
+        t = N // T
+        per = [0] * 8
+        for bi in range(t):
+            for bj in range(t):
+                per[(bi % P) * Q + bj % Q] += 3 * 8 * T * T
+        assert st["h2d_bytes"] == per
+        xk.reset_stats()
+        assert xk.dgemm_async("N", "N", N, N, N, 2.0, A, N, B, N, -1.0, C, N) == 0
+        xk.sync()
+        assert sum(xk.get_stats()["h2d_bytes"]) == 0
+        assert xk.memory_coherent_sync(N, N, C, N) == 0
+    finally:
+        xk.finalize()
+    assert np.array_equal(C, ref)

@@ -699,3 +699,34 @@ def test_shadow_only_when_it_fits(routine, G):
                                          mem_bytes=mem), [call])
         assert got == exp
         assert _uses_shadow(routine, got[0]) == expect, (mem, need)
+
+
+@pytest.mark.parametrize("grid,blk", [((2, 4), (1, 1)), ((4, 2), (1, 1)), ((2, 2), (2, 1)), ((1, 8), (1, 3))])
+def test_distribute_2dbc(grid, blk):
+    """xk_distribute_2dbc_async (SecIV-C): tile (bi, bj) lands on GPU
+    ((bi/mb) mod P) Q + ((bj/nb) mod Q), one H2D per tile; a following async DGEMM reads no
+    host tile (data on device), its operands forwarded between GPUs; bit-exact with the model."""
+    G, T, t = 8, 4, 6
+    N = T * t
+    P, Q = grid
+    mb, nb = blk
+    calls = [dict(routine=pm.DISTRIBUTE, m=N, n=N, C=X, ldc=N, grid=grid, mb=mb, nb=nb) for X in (A_ADDR, B_ADDR, C_ADDR)]
+    calls.append(gemm(m=N, n=N, k=N, lda=N, ldb=N, ldc=N, sync=False))
+    calls.append(dict(routine=pm.COHERENT, m=N, n=N, C=C_ADDR, ldc=N))
+    got, exp = both(uniform(G), dict(topo="ranked", optimistic=True, window=2, tile=T), calls)
+    assert got == exp
+    for recs in got[:3]:
+        assert len(recs) == t * t and all(r[1] == pm.H2D for r in recs)
+        for r in recs:
+            assert r[7] == ((r[3] // mb) % P) * Q + (r[4] // nb) % Q
+    assert not any(r[1] == pm.H2D for r in got[3])
+    assert sum(1 for r in got[4] if r[1] == pm.D2H) == t * t
+
+
+def test_distribute_rejects_bad_grid():
+    s = xk.PlanSession(uniform(4), tile=4)
+    with pytest.raises(xk.XKError):
+        s.call(xk.make_call(routine=pm.DISTRIBUTE, m=8, n=8, C=A_ADDR, ldc=8, grid=(3, 2), mb=1, nb=1))
+    with pytest.raises(xk.XKError):
+        s.call(xk.make_call(routine=pm.DISTRIBUTE, m=8, n=8, C=A_ADDR, ldc=8, grid=(2, 2), mb=0, nb=1))
+    s.close()
