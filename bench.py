@@ -318,6 +318,7 @@ def share_inputs(N, rank, ws):
     paths, base = obj[0]
     mats = [xk.shared_matrix(p, N, N, create=False) for p in paths]
     if rank == 0:
+        inputs.set_threads(len(os.sched_getaffinity(0)))  # torchrun sets OMP_NUM_THREADS=1
         for M, seed in zip(mats, (inputs.SEED_A, inputs.SEED_B, inputs.SEED_C)):
             inputs.uniform(seed, N, N, out=M)
     barrier(ws)
@@ -544,7 +545,12 @@ def run_xk(args, rank, ws):
            "mode": "A, B, C resident in HBM (prefetched, untimed); xk_dgemm_async + xk_sync per step, "
                    "C updated on the GPUs (no host traffic)"}
 
-    ablation = run_ablation(lib, A, B, C, ws, timer) if (G > 1 and not args.no_ablation and N >= 16384) else None
+    ablation = None
+    if G > 1 and not args.no_ablation and N >= 16384:
+        try:  # an extra: a failure here must not cost the main line
+            ablation = run_ablation(lib, A, B, C, ws, timer)
+        except Exception as e:  # noqa: BLE001
+            ablation = {"error": repr(e)[:300]}
     cpu = cpu_baseline(N, A, B, C) if (rank == 0 and not args.no_cpu_baseline and ws == 1) else None
     barrier(ws)
     if rank == 0:
@@ -553,7 +559,10 @@ def run_xk(args, rank, ws):
                 os.unlink(p)
     north = None
     if (G == 8 or args.north_star) and not args.no_north_star:
-        north = run_north_star(args, rank, ws, timer, N=args.ns_n)
+        try:
+            north = run_north_star(args, rank, ws, timer, N=args.ns_n)
+        except Exception as e:  # noqa: BLE001
+            north = {"error": repr(e)[:300]}
 
     timed = max(1, int(k_n))
     avg_ms = k_ms / timed

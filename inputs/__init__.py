@@ -30,6 +30,7 @@ def _lib():
         lib.xkgen_uniform.argtypes = [u64, i64, i64, dp, i64]
         lib.xkgen_int.argtypes = [u64, i64, i64, dp, i64, ctypes.c_int, ctypes.c_int]
         lib.xkgen_tri_dd.argtypes = [u64, i64, dp, i64, ctypes.c_int, ctypes.c_double]
+        lib.xkgen_set_threads.argtypes = [ctypes.c_int]
         _LIB = lib
     return _LIB
 
@@ -70,3 +71,8 @@ def tri_dd(seed, n, lower=True, ld=None, fill=0.0, out=None):
 
 def mix(z):
     return int(_lib().xkgen_mix(z))
+
+
+def set_threads(n):
+    """Threads of the (counter-based, thread-count independent) fills."""
+    _lib().xkgen_set_threads(int(n))

@@ -32,6 +32,15 @@ static inline double u01(uint64_t seed, uint64_t idx)
 
 uint64_t xkgen_mix(uint64_t z) { return mix(z); }
 
+/* threads of the fills (torchrun sets OMP_NUM_THREADS=1 in every rank; the one rank that
+ * generates the shared matrices asks for all of its cores) -- never affects the values */
+#ifdef _OPENMP
+#include <omp.h>
+void xkgen_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
+#else
+void xkgen_set_threads(int n) { (void)n; }
+#endif
+
 void xkgen_uniform(uint64_t seed, i64 m, i64 n, double *out, i64 ld)
 {
 #pragma omp parallel for schedule(static)

@@ -54,3 +54,16 @@ def test_tri_dd_structure():
     assert np.all((d >= 1) & (d < 2))
     off = L[np.tril_indices(n, -1)]
     assert np.all(np.abs(off) <= 1.0 / (2 * n))
+
+
+def test_fills_do_not_depend_on_thread_count():
+    """Counter-based: the same matrices at any OpenMP thread count (bench.py's rank 0 raises
+    it above torchrun's OMP_NUM_THREADS=1)."""
+    import numpy as np
+    outs = []
+    for n in (1, 3, 8):
+        inputs.set_threads(n)
+        outs.append((inputs.uniform(7, 123, 77), inputs.integers(8, 50, 61), inputs.tri_dd(9, 90)))
+    inputs.set_threads(1)
+    for a, b in zip(outs, outs[1:]):
+        assert all(np.array_equal(x, y) for x, y in zip(a, b))
