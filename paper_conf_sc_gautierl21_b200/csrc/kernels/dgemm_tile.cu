@@ -346,11 +346,19 @@ cudaError_t launch_dgemm_batch(bool ta, bool tb, TileBatch &b, cudaStream_t st) 
         static thread_local TmaBatch tb_;
         tb_.n = b.n;
         bool ok = true;
+        // the mn-contiguous operands go as 3D maps (one TMA box per stage) only if every
+        // task's can: the batch runs one kernel instance, 2D or 3D, for all of them
+        bool all3d = true;
+        for (int q = 0; q < b.n; ++q)
+            all3d = all3d && (ta || b.t[q].M % 16 == 0) && (!tb || b.t[q].N % 16 == 0);
         for (int q = 0; q < b.n && ok; ++q) {
             const TileTask &t = b.t[q];
             TmaTask &u = tb_.t[q];
-            ok = make_tma_operand(&u.mapA, t.A, ta ? t.K : t.M, ta ? t.M : t.K, t.lda, !ta, tma_bm()) &&
-                 make_tma_operand(&u.mapB, t.B, tb ? t.N : t.K, tb ? t.K : t.N, t.ldb, tb, tma_bn());
+            u.a3d = u.b3d = 0;
+            ok = make_tma_operand(&u.mapA, t.A, ta ? t.K : t.M, ta ? t.M : t.K, t.lda, !ta, tma_bm(),
+                                  all3d ? &u.a3d : nullptr) &&
+                 make_tma_operand(&u.mapB, t.B, tb ? t.N : t.K, tb ? t.K : t.N, t.ldb, tb, tma_bn(),
+                                  all3d ? &u.b3d : nullptr);
             u.C = t.C;
             u.ldc = t.ldc;
             u.M = t.M;

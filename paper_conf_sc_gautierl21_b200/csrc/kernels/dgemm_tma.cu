@@ -91,10 +91,25 @@ __device__ __forceinline__ uint32_t const_part(int base8, int x) {
     return (uint32_t)((base8 << 7) | (((x >> 1) & 7) << 4) | ((x & 1) << 3));
 }
 
-template <bool MN_CONTIG, int BMN>
+__device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap *map, int c0, int c1, int c2,
+                                            uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];\n" ::"r"(dst),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(bar)
+        : "memory");
+}
+
+// One stage of an operand.  mn-contiguous: BMN/16 boxes of 16(mn) x 16(k) -- as ONE 3D box
+// (16 mn, 16 k, BMN/16 chunks of 16 mn) when the map is 3D (same shared-memory image: chunk
+// q at q * 2048, rows = k, 128-byte swizzle per row), else one 2D box per chunk.
+template <bool MN_CONTIG, int BMN, bool D3>
 __device__ __forceinline__ void issue_operand(uint32_t dst, const CUtensorMap *map, int mn0, int k0,
                                               uint32_t bar) {
     if (MN_CONTIG) {
+        if (D3) {
+            tma_load_3d(dst, map, 0, k0, mn0 >> 4, bar);
+            return;
+        }
 #pragma unroll
         for (int q = 0; q < BMN / 16; ++q) tma_load_2d(dst + q * 2048, map, mn0 + 16 * q, k0, bar);
     } else {
@@ -102,7 +117,7 @@ __device__ __forceinline__ void issue_operand(uint32_t dst, const CUtensorMap *m
     }
 }
 
-template <bool TA, bool TB>
+template <bool TA, bool TB, bool D3>
 __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_constant__ TmaBatch batch) {
     constexpr bool A_MN = !TA;  // op(A) M x K: 'N' -> m contiguous
     constexpr bool B_MN = TB;   // op(B) K x N: 'T' -> n contiguous
@@ -151,8 +166,8 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
         const int s = kb % STAGES;
         const uint32_t dst = sbase + s * STAGE_BYTES;
         mbar_expect_tx(full(s), STAGE_BYTES);
-        issue_operand<A_MN, BM>(dst, &t.mapA, m0, kb * BK, full(s));
-        issue_operand<B_MN, BN>(dst + A_BYTES, &t.mapB, n0, kb * BK, full(s));
+        issue_operand<A_MN, BM, D3>(dst, &t.mapA, m0, kb * BK, full(s));
+        issue_operand<B_MN, BN, D3>(dst + A_BYTES, &t.mapB, n0, kb * BK, full(s));
     };
     if (tid == 0)
         for (int kb = 0; kb < STAGES && kb < KB; ++kb) produce(kb);
@@ -300,10 +315,31 @@ EncodeTiledFn encode_fn() {
 // Tensor map of a stored column-major operand (rows x cols, ld) for the TMA kernel.
 // mn_contig: the contiguous dimension is m/n (box 16 x 16); else it is k (box 16 x bmn).
 bool make_tma_operand(CUtensorMap *map, const double *X, int64_t rows, int64_t cols, int64_t ld,
-                      bool mn_contig, int bmn) {
+                      bool mn_contig, int bmn, int *is3d) {
     EncodeTiledFn fn = encode_fn();
     if (!fn) return false;
     if (((uintptr_t)X & 15) || ((ld * 8) & 15) || rows <= 0 || cols <= 0) return false;
+    if (is3d) *is3d = 0;
+    static int use3d = -1;
+    if (use3d < 0) {
+        const char *e = getenv("XK_TMA3D");
+        use3d = (e && *e == '0') ? 0 : 1;
+    }
+    if (mn_contig && is3d && use3d && rows % 16 == 0) {
+        // the same operand as (16 rows in a chunk, cols, rows/16 chunks): one box of
+        // 16 x 16 x bmn/16 per stage instead of bmn/16 boxes (every chunk in bounds)
+        cuuint64_t dims3[3] = {16u, (cuuint64_t)cols, (cuuint64_t)(rows / 16)};
+        cuuint64_t strides3[2] = {(cuuint64_t)(ld * 8), 128u};
+        cuuint32_t box3[3] = {16u, 16u, (cuuint32_t)(bmn / 16)};
+        cuuint32_t estr3[3] = {1u, 1u, 1u};
+        CUresult r3 = fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double *>(X), dims3, strides3, box3,
+                         estr3, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r3 == CUDA_SUCCESS) {
+            *is3d = 1;
+            return true;
+        }
+    }
     cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
     cuuint64_t strides[1] = {(cuuint64_t)(ld * 8)};
     cuuint32_t box[2] = {16u, mn_contig ? 16u : (cuuint32_t)bmn};
@@ -333,7 +369,7 @@ cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st) {
     }
     b.cta_start[b.n] = total;
     if (total == 0) return cudaSuccess;
-    static unsigned attr_set[4] = {0, 0, 0, 0};  // per (ta, tb) kernel, one bit per device
+    static unsigned attr_set[8] = {0, 0, 0, 0, 0, 0, 0, 0};  // per kernel instance, one bit per device
     auto go = [&](void (*kern)(TmaBatch), int which) -> cudaError_t {
         int dev = 0;
         cudaGetDevice(&dev);
@@ -345,10 +381,18 @@ cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st) {
         kern<<<total, NTHREADS, smem, st>>>(b);
         return cudaGetLastError();
     };
-    if (!ta && !tb) return go(dgemm_tma_kernel<false, false>, 0);
-    if (!ta && tb) return go(dgemm_tma_kernel<false, true>, 1);
-    if (ta && !tb) return go(dgemm_tma_kernel<true, false>, 2);
-    return go(dgemm_tma_kernel<true, true>, 3);
+    // 3D maps for the mn-contiguous operands only if every task of the batch has them (the
+    // caller builds all of a batch's maps 2D or all 3D; a mixed batch is an error)
+    bool d3 = true, any3 = false;
+    for (int q = 0; q < b.n; ++q) {
+        d3 = d3 && (ta || b.t[q].a3d) && (!tb || b.t[q].b3d);
+        any3 = any3 || b.t[q].a3d || b.t[q].b3d;
+    }
+    if (any3 && !d3) return cudaErrorInvalidValue;
+    if (!ta && !tb) return d3 ? go(dgemm_tma_kernel<false, false, true>, 4) : go(dgemm_tma_kernel<false, false, false>, 0);
+    if (!ta && tb) return d3 ? go(dgemm_tma_kernel<false, true, true>, 5) : go(dgemm_tma_kernel<false, true, false>, 1);
+    if (ta && !tb) return go(dgemm_tma_kernel<true, false, false>, 2);
+    return d3 ? go(dgemm_tma_kernel<true, true, true>, 7) : go(dgemm_tma_kernel<true, true, false>, 3);
 }
 
 }  // namespace xk

@@ -32,6 +32,7 @@ struct TileBatch {
 // TMA variant (dgemm_tma.cu): operands described by tensor maps (128-byte swizzle).
 struct TmaTask {
     CUtensorMap mapA, mapB;  // stored A / B tiles (make_tma_operand)
+    int a3d = 0, b3d = 0;    // mn-contiguous operand mapped as a 3D tensor: one box per stage
     double *C;
     int64_t ldc, M, N, K;
     double alpha, beta;
@@ -48,7 +49,7 @@ struct TmaBatch {
     TmaTask t[kMaxTmaBatch];
 };
 bool make_tma_operand(CUtensorMap *map, const double *X, int64_t rows, int64_t cols, int64_t ld,
-                      bool mn_contig, int bmn);
+                      bool mn_contig, int bmn, int *is3d = nullptr);
 int tma_bm();
 int tma_bn();
 cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st);

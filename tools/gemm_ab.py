@@ -15,21 +15,22 @@ import paper_conf_sc_gautierl21_b200 as xk  # noqa: E402
 N = int(os.environ.get("N", 32768))
 REPS = int(os.environ.get("REPS", 3))
 tiles = [int(t) for t in os.environ.get("TILES", "1024,2048,4096").split(",")]
+TA, TB = os.environ.get("TRANS", "NN")
 A, B, C = inputs.uniform(1, N, N), inputs.uniform(2, N, N), inputs.uniform(3, N, N)
-out = {"N": N, "env": {k: v for k, v in os.environ.items() if k.startswith("XK_")}}
+out = {"N": N, "trans": TA + TB, "env": {k: v for k, v in os.environ.items() if k.startswith("XK_")}}
 for T in tiles:
     xk.init(ngpus=1, tile=T, probe=False)
     for X in (A, B, C):
         xk.register(X)
         xk.memory_prefetch_async(N, N, X, N)
     xk.sync()
-    xk.dgemm_async("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
+    xk.dgemm_async(TA, TB, N, N, N, 1.5, A, N, B, N, -0.75, C, N)
     xk.sync()
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
     e0.record()
     for _ in range(REPS):
-        xk.dgemm_async("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
+        xk.dgemm_async(TA, TB, N, N, N, 1.5, A, N, B, N, -0.75, C, N)
         xk.sync()
     torch.cuda.synchronize()
     e1.record()
@@ -37,7 +38,7 @@ for T in tiles:
     ms = e0.elapsed_time(e1) / REPS
     xk.reset_stats()
     xk.set_kernel_timing(True)
-    xk.dgemm_async("N", "N", N, N, N, 1.5, A, N, B, N, -0.75, C, N)
+    xk.dgemm_async(TA, TB, N, N, N, 1.5, A, N, B, N, -0.75, C, N)
     xk.sync()
     st = xk.get_stats()
     xk.set_kernel_timing(False)
