@@ -18,7 +18,7 @@ def num(name, scale_to=None):
     val, unit = get[name]
     x = float(val.replace(",", ""))
     mult = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "msecond": 1e-3, "usecond": 1e-6, "nsecond": 1e-9,
-            "second": 1.0}
+            "second": 1.0, "ms": 1e-3, "us": 1e-6, "ns": 1e-9, "s": 1.0}
     return x * mult.get(unit, 1.0) if scale_to else x
 
 
