@@ -409,6 +409,9 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
     // to the member furthest below its quota.  When another requester asks first, the tile is
     // pulled to its designated GPU and forwarded from there (store-and-forward over NVLink).
     std::vector<int> puller(pending.size(), -1);
+    std::vector<int> slot_set(pending.size(), -1);   // shared requester set of a host-only slot
+    std::vector<std::vector<int64_t>> quota;         // per set: host tiles each member may still carry
+    std::vector<uint32_t> set_mask;
     if (flags_.optimistic && flags_.topo != XK_TOPO_HOME && G > 1) {
         std::vector<uint32_t> mask(pending.size(), 0);
         std::vector<int> order;  // slots in first-appearance order
@@ -449,23 +452,28 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
             count[it->second]++;
         }
         if (!sets.empty()) {
-            std::vector<std::vector<int64_t>> quota = balance_quotas(G, sets, count, forced);
-            std::vector<std::vector<int64_t>> given(sets.size(), std::vector<int64_t>(G, 0));
-            for (int s : order) {
-                if (puller[s] >= 0 || !host_only(s)) continue;
-                const int id = set_id[mask[s]];
-                const auto &q = quota[id];
-                auto &a = given[id];
-                int best = -1;  // least a/q among members with quota left (ties: lowest id)
-                for (int g = 0; g < G; ++g) {
-                    if (!(mask[s] >> g & 1) || a[g] >= q[g]) continue;
-                    if (best < 0 || a[g] * q[best] < a[best] * q[g]) best = g;
-                }
-                a[best]++;
-                puller[s] = best;
-            }
+            quota = balance_quotas(G, sets, count, forced);
+            for (int s : order)
+                if (puller[s] < 0 && host_only(s)) slot_set[s] = set_id[mask[s]];
+            set_mask = sets;
         }
     }
+    // the designated GPU of a shared tile is chosen at its first request (R16): the requester
+    // itself while its quota in that set lasts (no extra hop), else the member with the most
+    // quota left (ties: lowest id)
+    auto designate = [&](int slot, int d) {
+        const int id = slot_set[slot];
+        auto &q = quota[id];
+        if (q[d] > 0) {
+            q[d]--;
+            return d;
+        }
+        int best = -1;
+        for (int g = 0; g < G; ++g)
+            if ((set_mask[id] >> g & 1) && q[g] > 0 && (best < 0 || q[g] > q[best])) best = g;
+        q[best]--;
+        return best;
+    };
     // last writer per output tile
     std::unordered_map<int, size_t> last;
     for (size_t q = 0; q < tasks.size(); ++q) {
@@ -541,6 +549,7 @@ int Planner::run_tasks(std::vector<Task> &tasks, bool sync, std::vector<Rec> &ou
         for (size_t p = 0; p < t.in.size(); ++p) {
             const Input &in = t.in[p];
             Entry &e = entries_[in.key];
+            if (slot_set[in.cnt] >= 0 && puller[in.cnt] < 0) puller[in.cnt] = designate(in.cnt, d);
             const int pl = puller[in.cnt];
             if (pl >= 0 && pl != d && !(e.gpu[d].present && e.gpu[d].ver == in.ver)) {
                 // R16: the first host read of this tile goes to its designated GPU

@@ -584,7 +584,7 @@ class Model:
         for t in last.values():
             t["last"] = True
         # R16 balance-aware first host pull (FULL mode): who carries each host-only input
-        puller = {}
+        puller, lazy = {}, {}
         if self.opt and self.mode != HOME and self.G > 1:
             req, order = {}, []
             for t in tasks:
@@ -615,17 +615,19 @@ class Model:
                 shared.append(key)
             if sets:
                 quota = min_max_quotas(self.G, sets, [count[s] for s in sets], forced)
-                given = {s: [0] * self.G for s in sets}
                 for key in shared:
-                    gs = frozenset(req[key][2])
-                    q, a = quota[sets.index(gs)], given[gs]
-                    cands = [g for g in sorted(gs) if a[g] < q[g]]
-                    best = cands[0]
-                    for g in cands[1:]:
-                        if a[g] * q[best] < a[best] * q[g]:
-                            best = g
-                    a[best] += 1
-                    puller[key] = best
+                    lazy[key] = quota[sets.index(frozenset(req[key][2]))]
+
+        def designate(key, d):
+            """At the first request: the requester while its quota in the set lasts, else the
+            member with the most quota left (ties: lowest id)."""
+            q = lazy.pop(key)
+            if q[d] > 0:
+                q[d] -= 1
+                return d
+            best = max((g for g in range(self.G) if q[g] > 0), key=lambda g: (q[g], -g))
+            q[best] -= 1
+            return best
         lists = [[] for _ in range(self.G)]
         for t in tasks:
             lists[t["gpu"]].append(t)
@@ -660,6 +662,8 @@ class Model:
             ready_at = 0
             for p, (tl, v, operand) in enumerate(t["ins"]):
                 c = tl.gpus.get(d)
+                if (id(tl), v) in lazy:
+                    puller[(id(tl), v)] = designate((id(tl), v), d)
                 pl = puller.get((id(tl), v))
                 if (pl is not None and pl != d and (c is None or c.ver != v)
                         and not any(x.ver == v for x in tl.gpus.values())):

@@ -11,8 +11,9 @@ MODES = [("full", "ranked", True), ("no_opt", "ranked", False), ("no_opt_topo", 
 boxes = {
     # DGX-1: Fig. 2 GPU matrix; host links PCIe Gen3 x16 shared by 2 GPUs -> ~6 GB/s each
     "dgx1_v100": (with_host(fig2(), host=6000), 7000000),
-    # 8x B200: 55 GB/s PCIe Gen5 per GPU (measured), ~700 GB/s CE peer copies, 35 TF tile rate (measured)
-    "hgx_b200": (uniform(8, peer=700000, host=55000), 35000000),
+    # 8x B200: 55 GB/s PCIe Gen5 per GPU (measured), ~700 GB/s CE peer copies, 35.8 TF tile rate
+    # (round-2 grouped launch, measured)
+    "hgx_b200": (uniform(8, peer=700000, host=55000), 35800000),
 }
 out = {}
 for box, (bw, rate) in boxes.items():
@@ -24,7 +25,12 @@ for box, (bw, rate) in boxes.items():
             recs = xk.plan_dump(call, bw, rate_mflops=rate, topo=topo, optimistic=opt, tile=T, cap=1 << 18)
             t = max(r[12] for r in recs) * 1e-9
             h2d = sum(r[13] for r in recs if r[1] == 0) / 1e9
-            row[name] = {"pred_tflops": round(2.0 * N ** 3 / t / 1e12, 2), "h2d_GB": round(h2d, 2)}
+            per = [0] * 8
+            for r in recs:
+                if r[1] == 0:
+                    per[r[7]] += r[13]
+            row[name] = {"pred_tflops": round(2.0 * N ** 3 / t / 1e12, 2), "h2d_GB": round(h2d, 2),
+                         "h2d_max_over_mean": round(max(per) / (sum(per) / 8), 3)}
         out["%s_N%d" % (box, N)] = row
         print(box, N, json.dumps(row))
 # the north-star configuration (BASELINE configs[4]): N=65536 on 8x B200, tile sweep, full
