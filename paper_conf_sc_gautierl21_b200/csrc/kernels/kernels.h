@@ -22,7 +22,7 @@ struct TileTask {
 
 // A batch of independent tile tasks launched as one grid (grouped GEMM); passed by value
 // as a __grid_constant__ kernel parameter (32 * 88 + 136 bytes < 4 KB).
-constexpr int kMaxBatch = 64;
+constexpr int kMaxBatch = 32;
 struct TileBatch {
     int n = 0;
     int cta_start[kMaxBatch + 1] = {};
@@ -41,7 +41,7 @@ struct TmaTask {
     int64_t ldc2;
     double beta2;
 };
-constexpr int kMaxTmaBatch = 64;
+constexpr int kMaxTmaBatch = 16;
 struct TmaBatch {
     int n = 0;
     int group_m = 16;  // CTA raster: m-blocks per group (L2 reuse); 0 = column-major raster
