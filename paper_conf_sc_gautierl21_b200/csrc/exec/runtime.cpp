@@ -1299,66 +1299,70 @@ int Runtime::probe_host_links(int64_t bytes_per_gpu) {
         }
         bytes /= 2;
     }
-    for (size_t q = 0; q < n; ++q) {  // touch the pages (first-touch cost outside the timing)
-        std::memset(hin[q], 1, bytes);
-        std::memset(hout[q], 0, bytes);
-        cudaSetDevice(devs_[mine[q]].phys);
-        cudaMemset(din[q], 0, bytes);
-        cudaMemset(dout[q], 0, bytes);
-    }
-    auto sync_mine = [&]() -> int {
+    // the measurement; on any failure the buffers are still released below
+    auto measure = [&]() -> int {
+        for (size_t q = 0; q < n; ++q) {  // touch the pages (first-touch cost outside the timing)
+            std::memset(hin[q], 1, bytes);
+            std::memset(hout[q], 0, bytes);
+            cudaSetDevice(devs_[mine[q]].phys);
+            cudaMemset(din[q], 0, bytes);
+            cudaMemset(dout[q], 0, bytes);
+        }
+        auto sync_mine = [&]() -> int {
+            for (size_t q = 0; q < n; ++q) {
+                Device &d = devs_[mine[q]];
+                XK_CK(cudaStreamSynchronize(d.h2d));
+                XK_CK(cudaStreamSynchronize(d.d2h));
+            }
+            return XK_OK;
+        };
         for (size_t q = 0; q < n; ++q) {
-            Device &d = devs_[mine[q]];
-            XK_CK(cudaStreamSynchronize(d.h2d));
-            XK_CK(cudaStreamSynchronize(d.d2h));
+            XK_CK(cudaSetDevice(devs_[mine[q]].phys));
+            XK_CK(cudaDeviceSynchronize());
+        }
+        for (int pat = 0; pat < 3; ++pat) {  // 0 H2D, 1 D2H, 2 both
+            double best = 1e300;
+            for (int rep = 0; rep < 3; ++rep) {
+                if (rank_mode_ && !sess_->barrier(300.0)) {
+                    set_error("rank mode: a peer failed during the host-link probe");
+                    return XK_ERR_CUDA;
+                }
+                auto t0 = std::chrono::steady_clock::now();
+                for (size_t q = 0; q < n; ++q) {
+                    Device &d = devs_[mine[q]];
+                    XK_CK(cudaSetDevice(d.phys));
+                    if (pat != 1) XK_CK(cudaMemcpyAsync(din[q], hin[q], bytes, cudaMemcpyHostToDevice, d.h2d));
+                    if (pat != 0) XK_CK(cudaMemcpyAsync(hout[q], dout[q], bytes, cudaMemcpyDeviceToHost, d.d2h));
+                }
+                if ((rc = sync_mine())) return rc;
+                double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+                if (rep > 0) best = std::min(best, ms);
+            }
+            double tot_bytes = (double)bytes * (pat == 2 ? 2 : 1) * (double)n, tmax = best;
+            if (rank_mode_) {  // aggregate over ranks: all bytes / the slowest rank's time
+                SessionRank &me = sess_->hdr()->rank[rank_];
+                me.host_probe_ms = best;
+                me.host_probe_bytes = (int64_t)bytes;
+                if (!sess_->barrier(300.0)) {
+                    set_error("rank mode: a peer failed during the host-link probe");
+                    return XK_ERR_CUDA;
+                }
+                tot_bytes = 0;
+                tmax = 0;
+                for (int g = 0; g < G; ++g) {
+                    const SessionRank &r = sess_->hdr()->rank[g];
+                    tot_bytes += (double)r.host_probe_bytes * (pat == 2 ? 2 : 1);
+                    tmax = std::max(tmax, r.host_probe_ms);
+                }
+            }
+            host_all_MBps[pat] = (int64_t)(tot_bytes / (tmax * 1e-3) / 1e6);
         }
         return XK_OK;
     };
-    for (size_t q = 0; q < n; ++q) {
-        XK_CK(cudaSetDevice(devs_[mine[q]].phys));
-        XK_CK(cudaDeviceSynchronize());
-    }
-    for (int pat = 0; pat < 3; ++pat) {  // 0 H2D, 1 D2H, 2 both
-        double best = 1e300;
-        for (int rep = 0; rep < 3; ++rep) {
-            if (rank_mode_ && !sess_->barrier(300.0)) {
-                release();
-                set_error("rank mode: a peer failed during the host-link probe");
-                return XK_ERR_CUDA;
-            }
-            auto t0 = std::chrono::steady_clock::now();
-            for (size_t q = 0; q < n; ++q) {
-                Device &d = devs_[mine[q]];
-                XK_CK(cudaSetDevice(d.phys));
-                if (pat != 1) XK_CK(cudaMemcpyAsync(din[q], hin[q], bytes, cudaMemcpyHostToDevice, d.h2d));
-                if (pat != 0) XK_CK(cudaMemcpyAsync(hout[q], dout[q], bytes, cudaMemcpyDeviceToHost, d.d2h));
-            }
-            if ((rc = sync_mine())) {
-                release();
-                return rc;
-            }
-            double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
-            if (rep > 0) best = std::min(best, ms);
-        }
-        double tot_bytes = (double)bytes * (pat == 2 ? 2 : 1) * (double)n, tmax = best;
-        if (rank_mode_) {  // aggregate over ranks: all bytes / the slowest rank's time
-            SessionRank &me = sess_->hdr()->rank[rank_];
-            me.host_probe_ms = best;
-            me.host_probe_bytes = (int64_t)bytes;
-            if (!sess_->barrier(300.0)) {
-                release();
-                set_error("rank mode: a peer failed during the host-link probe");
-                return XK_ERR_CUDA;
-            }
-            tot_bytes = 0;
-            tmax = 0;
-            for (int g = 0; g < G; ++g) {
-                const SessionRank &r = sess_->hdr()->rank[g];
-                tot_bytes += (double)r.host_probe_bytes * (pat == 2 ? 2 : 1);
-                tmax = std::max(tmax, r.host_probe_ms);
-            }
-        }
-        host_all_MBps[pat] = (int64_t)(tot_bytes / (tmax * 1e-3) / 1e6);
+    rc = measure();
+    if (rc) {
+        release();
+        return rc;
     }
     host_probe_bytes = (int64_t)bytes;
     release();

@@ -65,7 +65,7 @@ def main():
         for name, (rows, cols) in list(mats.items()):
             mats[name] = xk.shared_matrix(os.path.join(args.dir, name), rows, cols, create=False)
 
-    if args.case in ("gemm", "compose", "dod"):
+    if args.case in ("gemm", "compose", "dod", "distribute"):
         mat("A", N, N, lambda M: inputs.integers(1, N, N, out=M))
         mat("B", N, N, lambda M: inputs.integers(2, N, N, out=M))
         mat("C", N, N, lambda M: inputs.integers(3, N, N, out=M))
@@ -126,6 +126,17 @@ def main():
         assert xk.dgemm_async("N", "N", N, N, N, 1.0, m["A"], N, m["B"], N, -1.0, m["C"], N) == 0
         xk.sync()
         xk.memory_coherent_sync(N, N, m["C"], N)
+    elif args.case == "distribute":
+        # the paper's data-on-device: 2D block-cyclic on a (1, world) grid,
+        # transposed to the library's (world, 1) owner grid: every task reads peer tiles
+        for name in ("A", "B", "C"):
+            xk.distribute_2dbc_async(N, N, m[name], N, 1, args.world)
+        xk.sync()
+        out["dist_h2d"] = xk.get_stats()["h2d_bytes"][r]
+        xk.reset_stats()
+        assert xk.dgemm_async("N", "N", N, N, N, 1.0, m["A"], N, m["B"], N, -1.0, m["C"], N) == 0
+        xk.sync()
+        xk.memory_coherent_sync(N, N, m["C"], N)
     elif args.case == "big":
         # bench.py's launch configuration (alpha, beta, tile) on exact-integer inputs
         assert xk.dgemm("N", "N", N, N, N, 1.5, m["A"], N, m["B"], N, -0.75, m["C"], N) == 0
@@ -152,7 +163,7 @@ def main():
             refE = np.zeros((N, N), order="F")
             oracle.dgemm("T", "N", N, N, N, 1.0, c["A"], ref, 0.0, refE)
             check("E bitwise", np.array_equal(np.asarray(m["E"]), refE))
-        elif args.case == "dod":
+        elif args.case in ("dod", "distribute"):
             ref = c["C"].copy(order="F")
             oracle.dgemm("N", "N", N, N, N, 1.0, c["A"], c["B"], -1.0, ref)
             check("C bitwise", np.array_equal(np.asarray(m["C"]), ref))

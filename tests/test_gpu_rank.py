@@ -131,6 +131,20 @@ def test_rank_mode_data_on_device_and_probe():
         assert all(bw[s][d] > 0 for s in range(3) for d in range(3))
 
 
+def test_rank_mode_distribute_2dbc():
+    """xk_distribute_2dbc_async in rank mode: each process loads the tiles of its grid column
+    (block-cyclic on a 1 x world grid, (1,1) blocks); the DGEMM then moves no host byte, its
+    operands pulled from the peers' arenas; bitwise vs the oracle."""
+    world, N, T = 4, 1024, 256
+    outs = run_ranks(world, "distribute", N, T)
+    t = N // T
+    for o in outs:
+        cols = sum(1 for bj in range(t) if bj % world == o["rank"])
+        assert o["dist_h2d"] == 3 * t * cols * 8 * T * T
+        assert o["stats"]["h2d_bytes"] == 0
+    assert sum(o["stats"]["p2p_in_bytes"] for o in outs) > 0
+
+
 def test_rank_mode_blas3():
     run_ranks(4, "blas3", 700, 128)
 
