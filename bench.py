@@ -472,7 +472,10 @@ def run_north_star(args, rank, ws, timer, N=65536, T=4096, steps=2):
     try:
         lib = Lib(args, rank, ws, base or "")
         xk = lib.init((A, B, C), T)
-        xk.probe_host_links(1 << 30)
+        try:
+            xk.probe_host_links(1 << 30)
+        except xk.XKError:
+            pass
         topo = xk.get_topology()
         r = timed_host_resident(xk, A, B, C, N, T, steps, 1, ws, timer)
         xk.finalize()
@@ -499,8 +502,12 @@ def run_xk(args, rank, ws):
     A, B, C, paths, base = share_inputs(N, rank, ws)
     lib = Lib(args, rank, ws, base)
     xk = lib.init((A, B, C), T)
-    # host links with every GPU copying at once (untimed set-up, like a1)
-    xk.probe_host_links(args.host_probe_mib << 20)
+    # host links with every GPU copying at once (untimed set-up, like a1); a
+    # failure (collective in rank mode) leaves the e2e roofline on the per-GPU probe
+    try:
+        xk.probe_host_links(args.host_probe_mib << 20)
+    except xk.XKError as e:
+        print("bench: concurrent host-link probe failed: %s" % e, file=sys.stderr)
     topo = xk.get_topology()
     timer = DevTimer()
     clocks = ClockSampler()

@@ -1268,33 +1268,60 @@ int Runtime::probe_host_links(int64_t bytes_per_gpu) {
     const size_t n = mine.size();
     std::vector<void *> hin(n, nullptr), hout(n, nullptr), din(n, nullptr), dout(n, nullptr);
     size_t bytes = (size_t)bytes_per_gpu;
+    // rank mode: the device side of the probe lives in the free top of this rank's tile arena
+    // (the arena holds most of the device memory; a cudaMalloc next to it may not fit)
+    const bool in_arena = rank_mode_;
     auto release = [&]() {
         for (size_t q = 0; q < n; ++q) {
             if (hin[q]) cudaFreeHost(hin[q]);
             if (hout[q]) cudaFreeHost(hout[q]);
             cudaSetDevice(devs_[mine[q]].phys);
-            if (din[q]) cudaFree(din[q]);
-            if (dout[q]) cudaFree(dout[q]);
+            if (!in_arena && din[q]) cudaFree(din[q]);
+            if (!in_arena && dout[q]) cudaFree(dout[q]);
             hin[q] = hout[q] = din[q] = dout[q] = nullptr;
         }
         cudaGetLastError();
         cur_dev_ = -1;
     };
-    // allocate (halving on failure; rank mode: every rank must end with the same size, so a
-    // rank that cannot allocate aborts the session instead of silently probing less)
+    // allocate, halving on failure down to 64 MiB; rank mode: collectively (every rank must
+    // probe the same size): each posts whether it could allocate, all halve if one could not
     for (;;) {
         bool ok = true;
         for (size_t q = 0; q < n && ok; ++q) {
             ok = cudaHostAlloc(&hin[q], bytes, cudaHostAllocPortable) == cudaSuccess &&
                  cudaHostAlloc(&hout[q], bytes, cudaHostAllocPortable) == cudaSuccess &&
-                 cudaSetDevice(devs_[mine[q]].phys) == cudaSuccess &&
-                 cudaMalloc(&din[q], bytes) == cudaSuccess && cudaMalloc(&dout[q], bytes) == cudaSuccess;
+                 cudaSetDevice(devs_[mine[q]].phys) == cudaSuccess;
+            if (ok && in_arena) {
+                const Device &d = devs_[mine[q]];
+                const int64_t top = d.arena_bytes - 2 * (int64_t)bytes;
+                ok = top >= round_up(d.arena_top, 1024);
+                if (ok) {
+                    din[q] = d.arena + top;
+                    dout[q] = d.arena + top + bytes;
+                }
+            } else if (ok) {
+                ok = cudaMalloc(&din[q], bytes) == cudaSuccess && cudaMalloc(&dout[q], bytes) == cudaSuccess;
+            }
+        }
+        if (rank_mode_) {
+            SessionRank &me = sess_->hdr()->rank[rank_];
+            me.host_probe_bytes = ok ? (int64_t)bytes : 0;
+            if (!sess_->barrier(300.0)) {
+                release();
+                set_error("rank mode: a peer failed during the host-link probe");
+                return XK_ERR_CUDA;
+            }
+            for (int g = 0; g < G; ++g) ok = ok && sess_->hdr()->rank[g].host_probe_bytes == (int64_t)bytes;
+            if (!sess_->barrier(300.0)) {  // everyone has read the flags before they change
+                release();
+                set_error("rank mode: a peer failed during the host-link probe");
+                return XK_ERR_CUDA;
+            }
         }
         if (ok) break;
         release();
-        if (rank_mode_ || bytes / 2 < ((size_t)64 << 20)) {
+        if (bytes / 2 < ((size_t)64 << 20)) {
             set_error("xk_probe_host_links: cannot allocate the probe buffers");
-            if (rank_mode_) sess_->abort();
             return XK_ERR_OOM;
         }
         bytes /= 2;
