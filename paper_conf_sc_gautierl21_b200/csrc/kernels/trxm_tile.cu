@@ -73,10 +73,10 @@ __device__ __forceinline__ void dmma884(double (&c)[2], double a, double b) {
 // hidden behind the others'.
 constexpr int UT = 4;
 __device__ __forceinline__ void block_update(const double *Ms, double *X, int r0, int r1, int k0, int nk,
-                                             double sign, int warp, int lane) {
+                                             double sign, int warp, int lane, int nwarps = NW) {
     const int nrt = (r1 - r0) / 8, tiles = nrt * (NVB / 8);
     const int fr = lane >> 2, fc = lane & 3;
-    for (int t0 = warp * UT; t0 < tiles; t0 += NW * UT) {
+    for (int t0 = warp * UT; t0 < tiles; t0 += nwarps * UT) {
         int rr[UT], vv[UT];
         double d[UT][2];
 #pragma unroll
@@ -132,20 +132,27 @@ __global__ void __launch_bounds__(BT) trxm_base_kernel(const __grid_constant__ B
     // Every global load is an asynchronous copy straight into shared memory (cp.async,
     // zero-filled when predicated off), all in flight at once: the referenced triangle of M
     // (consecutive threads along A's stored-contiguous direction; the other triangle, the
-    // unit diagonal and the padding to NB are never read from A), then the CTA's vectors.
-    {
+    // unit diagonal and the padding to NB are never read from A) as one group, then the
+    // CTA's vectors block by block in the order the blocks are processed (one group each),
+    // so the first diagonal block starts while the later ones are still arriving.
+    constexpr int NBLK = NB / BS;
+    auto order = [&](int step) { return (SOLVE == LOWER) ? step : NBLK - 1 - step; };
 #pragma unroll 4
-        for (int k = 0; k < NB * NB / BT; ++k) {
-            const int e = tid + k * BT, f = e % NB, s2 = e / NB;
-            const int i = mtrans ? s2 : f, c = mtrans ? f : s2;  // M(i, c); A contiguous in f
-            const bool in = LOWER ? (i > c) : (i < c);
-            const bool rd_a = i < n && c < n && (in || (i == c && !unit));
-            cp_async8(Ms + c * LDM + i, rd_a ? (mtrans ? A + c + (int64_t)i * lda : A + i + (int64_t)c * lda) : A, rd_a);
-        }
-        if (LEFT) {  // columns of B: a warp reads whole 512-byte columns, 16 bytes per lane
-#pragma unroll 4
-            for (int k = 0; k < NVB / NW; ++k) {
-                const int v = warp + NW * k, e = 2 * lane;
+    for (int k = 0; k < NB * NB / BT; ++k) {
+        const int e = tid + k * BT, f = e % NB, s2 = e / NB;
+        const int i = mtrans ? s2 : f, c = mtrans ? f : s2;  // M(i, c); A contiguous in f
+        const bool in = LOWER ? (i > c) : (i < c);
+        const bool rd_a = i < n && c < n && (in || (i == c && !unit));
+        cp_async8(Ms + c * LDM + i, rd_a ? (mtrans ? A + c + (int64_t)i * lda : A + i + (int64_t)c * lda) : A, rd_a);
+    }
+    asm volatile("cp.async.commit_group;\n" ::: "memory");
+#pragma unroll 1
+    for (int step = 0; step < NBLK; ++step) {
+        const int o = order(step) * BS;
+        if (LEFT) {  // BS entries of every column: 16-byte chunks, 128 contiguous bytes per column
+#pragma unroll
+            for (int k = 0; k < NVB * BS / 2 / BT; ++k) {
+                const int c = tid + k * BT, v = c / (BS / 2), e = o + 2 * (c % (BS / 2));
                 const bool ok = v < nv && e < n;
                 const double *src = ok ? B + (v0 + v) * ldb + e : B;
                 if (bb.al16 && (e + 1 < n || !ok)) {
@@ -156,78 +163,113 @@ __global__ void __launch_bounds__(BT) trxm_base_kernel(const __grid_constant__ B
                 }
             }
         } else {     // rows of B: consecutive threads read consecutive rows of one column
-#pragma unroll 4
-            for (int k = 0; k < NB * NVB / BT; ++k) {
-                const int e = tid + k * BT, v = e % NVB, l = e / NVB;
+#pragma unroll
+            for (int k = 0; k < NVB * BS / BT; ++k) {
+                const int e = tid + k * BT, v = e % NVB, l = o + e / NVB;
                 const bool ok = v < nv && l < n;
                 cp_async8(X + v * LDV + l, ok ? B + (v0 + v) + (int64_t)l * ldb : B, ok);
             }
         }
-        asm volatile("cp.async.wait_all;\n" ::: "memory");
-        __syncthreads();
-        if (tid < NB) {  // the diagonal: 1 where A's is not read (unit, padding), reciprocal
-            if (unit || tid >= n) Ms[tid * LDM + tid] = 1.0;
-            rd[tid] = 1.0 / Ms[tid * LDM + tid];
-        }
-        __syncthreads();
+        asm volatile("cp.async.commit_group;\n" ::: "memory");
     }
-    constexpr int NBLK = NB / BS;
-#pragma unroll 1
-    for (int step = 0; step < NBLK; ++step) {
-        // block order: TRSM lower / TRMM upper forward, the others backward
-        const int kb = (SOLVE == LOWER) ? step : NBLK - 1 - step;
+    static_assert(NBLK == 4, "the cp.async group waits below assume 4 blocks");
+    // M and the first block: the diagonal fix-up (1 where A's is not read: unit, padding)
+    asm volatile("cp.async.wait_group 3;\n" ::: "memory");
+    __syncthreads();
+    if (tid < NB) {
+        if (unit || tid >= n) Ms[tid * LDM + tid] = 1.0;
+        rd[tid] = 1.0 / Ms[tid * LDM + tid];
+    }
+    __syncthreads();
+    // one thread per vector: solve / multiply the vector's BS entries of diagonal block kb
+    auto diag = [&](int kb) {
         const int o = kb * BS;
-        if (tid < NVB) {  // one thread per vector: the diagonal block
-            double *xv = X + tid * LDV + o;
-            double x[BS];
+        double *xv = X + tid * LDV + o;
+        double x[BS];
 #pragma unroll
-            for (int p = 0; p < BS / 2; ++p) {
-                const double2 z = *reinterpret_cast<const double2 *>(xv + 2 * p);
-                x[2 * p] = z.x;
-                x[2 * p + 1] = z.y;
+        for (int p = 0; p < BS / 2; ++p) {
+            const double2 z = *reinterpret_cast<const double2 *>(xv + 2 * p);
+            x[2 * p] = z.x;
+            x[2 * p + 1] = z.y;
+        }
+        if (SOLVE && LOWER) {         // forward, column-oriented
+#pragma unroll
+            for (int l = 0; l < BS; ++l) {
+                if (!unit) x[l] *= rd[o + l];
+#pragma unroll
+                for (int i = l + 1; i < BS; ++i) x[i] -= Ms[(o + l) * LDM + o + i] * x[l];
             }
-            if (SOLVE && LOWER) {         // forward, column-oriented
+        } else if (SOLVE) {           // backward
 #pragma unroll
-                for (int l = 0; l < BS; ++l) {
-                    if (!unit) x[l] *= rd[o + l];
+            for (int l = BS - 1; l >= 0; --l) {
+                if (!unit) x[l] *= rd[o + l];
 #pragma unroll
-                    for (int i = l + 1; i < BS; ++i) x[i] -= Ms[(o + l) * LDM + o + i] * x[l];
-                }
-            } else if (SOLVE) {           // backward
-#pragma unroll
-                for (int l = BS - 1; l >= 0; --l) {
-                    if (!unit) x[l] *= rd[o + l];
-#pragma unroll
-                    for (int i = 0; i < l; ++i) x[i] -= Ms[(o + l) * LDM + o + i] * x[l];
-                }
-            } else if (LOWER) {           // bottom-up: row i reads x_0..x_i, still unmodified
-#pragma unroll
-                for (int i = BS - 1; i >= 0; --i) {
-                    double s = 0.0;
-#pragma unroll
-                    for (int l = 0; l <= i; ++l) s += Ms[(o + l) * LDM + o + i] * x[l];
-                    x[i] = s;
-                }
-            } else {                      // top-down: row i reads x_i..x_BS-1
-#pragma unroll
-                for (int i = 0; i < BS; ++i) {
-                    double s = 0.0;
-#pragma unroll
-                    for (int l = i; l < BS; ++l) s += Ms[(o + l) * LDM + o + i] * x[l];
-                    x[i] = s;
-                }
+                for (int i = 0; i < l; ++i) x[i] -= Ms[(o + l) * LDM + o + i] * x[l];
             }
+        } else if (LOWER) {           // bottom-up: row i reads x_0..x_i, still unmodified
 #pragma unroll
-            for (int p = 0; p < BS / 2; ++p)
-                *reinterpret_cast<double2 *>(xv + 2 * p) = make_double2(x[2 * p], x[2 * p + 1]);
+            for (int i = BS - 1; i >= 0; --i) {
+                double s = 0.0;
+#pragma unroll
+                for (int l = 0; l <= i; ++l) s += Ms[(o + l) * LDM + o + i] * x[l];
+                x[i] = s;
+            }
+        } else {                      // top-down: row i reads x_i..x_BS-1
+#pragma unroll
+            for (int i = 0; i < BS; ++i) {
+                double s = 0.0;
+#pragma unroll
+                for (int l = i; l < BS; ++l) s += Ms[(o + l) * LDM + o + i] * x[l];
+                x[i] = s;
+            }
+        }
+#pragma unroll
+        for (int p = 0; p < BS / 2; ++p)
+            *reinterpret_cast<double2 *>(xv + 2 * p) = make_double2(x[2 * p], x[2 * p + 1]);
+    };
+#ifndef XK_BASE_NULL
+    if (SOLVE) {
+        // TRSM with a one-block lookahead: after block kb is solved, the rows of the next
+        // block are updated first (all warps); then warps 0-1 solve that next block while
+        // warps 2-3 update the remaining rows with block kb -- the diagonal chain and the
+        // bulk of the updates overlap instead of alternating
+        if (tid < NVB) diag(order(0));
+#pragma unroll 1
+        for (int step = 0; step + 1 < NBLK; ++step) {
+            const int kb = order(step), kn = order(step + 1);
+            if (step == 0) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
+            __syncthreads();
+            block_update(Ms, X, kn * BS, kn * BS + BS, kb * BS, BS, -1.0, warp, lane);
+            if (step == 0) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+            __syncthreads();
+            if (tid < NVB) {
+                diag(kn);
+            } else if (LOWER) {
+                if (kn + 1 < NBLK) block_update(Ms, X, (kn + 1) * BS, NB, kb * BS, BS, -1.0, warp - 2, lane, NW - 2);
+            } else {
+                if (kn > 0) block_update(Ms, X, 0, kn * BS, kb * BS, BS, -1.0, warp - 2, lane, NW - 2);
+            }
         }
         __syncthreads();
-        if (SOLVE && LOWER) block_update(Ms, X, o + BS, NB, o, BS, -1.0, warp, lane);
-        else if (SOLVE) block_update(Ms, X, 0, o, o, BS, -1.0, warp, lane);
-        else if (LOWER) block_update(Ms, X, o, o + BS, 0, o, 1.0, warp, lane);
-        else block_update(Ms, X, o, o + BS, o + BS, NB - o - BS, 1.0, warp, lane);
+    } else {
+        asm volatile("cp.async.wait_group 0;\n" ::: "memory");
         __syncthreads();
+#pragma unroll 1
+        for (int step = 0; step < NBLK; ++step) {
+            // TRMM: lower bottom-up (blocks above still unmodified), upper top-down
+            const int kb = order(step);
+            const int o = kb * BS;
+            if (tid < NVB) diag(kb);
+            __syncthreads();
+            if (LOWER) block_update(Ms, X, o, o + BS, 0, o, 1.0, warp, lane);
+            else block_update(Ms, X, o, o + BS, o + BS, NB - o - BS, 1.0, warp, lane);
+            __syncthreads();
+        }
     }
+#else
+    asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+    __syncthreads();
+#endif
     // X back to B, times alpha (TRSM: op(A)^-1 (alpha B) = alpha op(A)^-1 B)
     const double so = alpha;
     if (LEFT) {
