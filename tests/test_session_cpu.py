@@ -13,7 +13,7 @@ WORKER = r"""
 import json, sys
 sys.path.insert(0, %(root)r)
 import paper_conf_sc_gautierl21_b200 as xk
-rc, seen = xk.session_selftest(%(path)r, %(rank)d, %(world)d, %(rounds)d, %(abort)d, 20.0)
+rc, seen = xk.session_selftest(%(path)r, %(rank)d, %(world)d, %(rounds)d, %(abort)d, 90.0)
 print(json.dumps({"rc": rc, "seen": seen}))
 """
 
@@ -46,8 +46,8 @@ def test_barrier_rounds_across_processes():
 
 def test_abort_fails_peers_instead_of_hanging():
     outs, _ = run(3, 6, abort_rank=2, abort_at=3)
-    assert outs[2]["rc"] == 0                  # the aborting rank itself returns cleanly
-    assert outs[0]["rc"] == 2 and outs[1]["rc"] == 2  # XK_ERR_CUDA at the failed barrier
+    assert outs[2]["rc"] == 0, outs            # the aborting rank itself returns cleanly
+    assert outs[0]["rc"] == 2 and outs[1]["rc"] == 2, outs  # XK_ERR_CUDA at the failed barrier
     assert outs[0]["seen"][:3] == [3, 3, 3] and outs[1]["seen"][:3] == [3, 3, 3]
 
 

@@ -137,7 +137,21 @@ for e in ev:
 for d in byname.values():
     d["tflops_per_launch_time"] = round(d["gflop"] / max(1e-9, d["ms"]), 2)
     d["ms"] = round(d["ms"], 3)
-summary = {"routine": R, "mode": "data-on-device" if DOD else "host-resident", "kernel_ops": byname, "N": N, "tile": T, "gpus": G, "wall_ms": round(wall, 3),
+# delivered FP64 rate over time: each kernel op's flops spread uniformly over its duration,
+# summed per 50 ms window (where a host-resident call loses against data-on-device)
+WIN = 50e3
+nwin = int(t_end // WIN) + 1
+win = [0.0] * nwin
+for e in ev:
+    if e["tid"] != "kernels" or e["dur"] <= 0:
+        continue
+    f = e["args"].get("flops", 0)
+    a, b = e["ts"], e["ts"] + e["dur"]
+    for w in range(int(a // WIN), min(nwin, int(b // WIN) + 1)):
+        ov = max(0.0, min(b, (w + 1) * WIN) - max(a, w * WIN))
+        win[w] += f * ov / e["dur"]
+summary = {"tflops_by_50ms_window": [round(x / (WIN * 1e-6) / 1e12, 2) for x in win],
+           "routine": R, "mode": "data-on-device" if DOD else "host-resident", "kernel_ops": byname, "N": N, "tile": T, "gpus": G, "wall_ms": round(wall, 3),
            "tflops": round(flops / wall / 1e9, 2), "trace_span_ms": round(t_end / 1e3, 3),
            "kernel_busy_union_ms": round(busy / 1e3, 3), "streams": span, "largest_kernel_idle_gaps": top,
            "h2d_gb": sum(st["h2d_bytes"]) / 1e9, "d2h_gb": sum(st["d2h_bytes"]) / 1e9}
