@@ -78,10 +78,10 @@ typedef struct xk_config {
     int64_t tile;         /* tile size T (0 = 2048) */
     int topo;             /* XK_TOPO_* (default RANKED) */
     int optimistic;       /* optimistic forwarding on (1, default) / off (0) */
-    int window;           /* planner prefetch window W in tasks (0 = 2) */
+    int window;           /* planner prefetch window W in tasks (0 = 4; Q17) */
     int kstreams;         /* kernel streams per GPU (0 = 2); plus 1 H2D, 1 D2H, 1 P2P-in */
     int probe;            /* 1 = time the (G+1)^2 link matrix at init (a1); 0 = defaults */
-    int64_t task_rate_mflops; /* planner's tile-task rate (0 = derived from the FP64 peak) */
+    int64_t task_rate_mflops; /* planner's tile-task rate (0 = measured at init on one grouped launch of 8 tile tasks; 35e6 without the probe) */
     /* ---- rank mode: one process per GPU.  `world` processes each call
      * xk_init with their own `rank` and the same `session`; process r drives logical GPU r
      * only.  Every process runs the same deterministic planner on the same calls, so all

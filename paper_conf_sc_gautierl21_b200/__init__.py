@@ -264,7 +264,7 @@ def _topo(bw, rate_mflops):
     return t
 
 
-def _flags(topo="ranked", optimistic=True, window=2, grid=(0, 0), tile=2048, mem_bytes=0):
+def _flags(topo="ranked", optimistic=True, window=4, grid=(0, 0), tile=2048, mem_bytes=0):
     f = _abi.Flags()
     f.mem_bytes = int(mem_bytes)
     f.topo = TOPO_NAMES[topo] if isinstance(topo, str) else int(topo)

@@ -112,7 +112,7 @@ void xk_config_default(xk_config_t *cfg) {
     if (topo && !std::strcmp(topo, "unranked")) cfg->topo = XK_TOPO_UNRANKED;
     if (topo && !std::strcmp(topo, "home")) cfg->topo = XK_TOPO_HOME;
     cfg->optimistic = env_int("XK_OPTIMISTIC", 1);
-    cfg->window = env_int("XK_WINDOW", 2);
+    cfg->window = env_int("XK_WINDOW", 4);
     cfg->kstreams = env_int("XK_KSTREAMS", 2);
     cfg->probe = env_int("XK_PROBE", 1);
 }

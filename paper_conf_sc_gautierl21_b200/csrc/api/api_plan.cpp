@@ -50,7 +50,7 @@ bool make_flags(const xk_flags_t *f, int G, Flags *out, std::string &err) {
     if (f) {
         F.topo = f->topo;
         F.optimistic = f->optimistic;
-        F.window = f->window > 0 ? f->window : 2;
+        F.window = f->window > 0 ? f->window : 4;
         F.T = f->tile > 0 ? f->tile : 2048;
         F.P = f->grid_p;
         F.Q = f->grid_q;

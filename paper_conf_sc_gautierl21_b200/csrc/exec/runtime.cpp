@@ -125,7 +125,7 @@ int Runtime::init(const xk_config_t &cfg) {
     // flags
     flags_.topo = cfg.topo;
     flags_.optimistic = cfg.optimistic;
-    flags_.window = cfg.window > 0 ? cfg.window : 2;
+    flags_.window = cfg.window > 0 ? cfg.window : 4;
     flags_.T = cfg.tile > 0 ? cfg.tile : 2048;
     flags_.P = cfg.grid_p;
     flags_.Q = cfg.grid_q;
@@ -258,25 +258,32 @@ int Runtime::probe_topology() {
             topo.bw[(size_t)s * N + d] = mbps(ms);
         }
     topo.bw[(size_t)G * N + G] = topo.bw[0];
-    // FP64 tile-task rate on GPU 0 (one T x T x T tile GEMM, T <= 2048)
+    // FP64 tile-task rate on GPU 0: one grouped launch of kRateTasks T x T x T tile GEMMs
+    // (T <= 2048), the form the executor launches them in -- a lone tile launch leaves part
+    // of the last wave idle and under-states the rate the planner's virtual time should use
     if (cfg_.task_rate_mflops <= 0) {
+        constexpr int kRateTasks = 8;
         int64_t T = std::min<int64_t>(flags_.T, 2048);
         size_t tb = (size_t)T * T * 8;
         double *a = nullptr, *b = nullptr, *c = nullptr;
         XK_CK(cudaSetDevice(devs_[0].phys));
         XK_CK(cudaMalloc(&a, tb));
         XK_CK(cudaMalloc(&b, tb));
-        XK_CK(cudaMalloc(&c, tb));
+        XK_CK(cudaMalloc(&c, tb * kRateTasks));
         XK_CK(cudaMemsetAsync(a, 0, tb, devs_[0].ks[0]));
         XK_CK(cudaMemsetAsync(b, 0, tb, devs_[0].ks[0]));
-        XK_CK(cudaMemsetAsync(c, 0, tb, devs_[0].ks[0]));
+        XK_CK(cudaMemsetAsync(c, 0, tb * kRateTasks, devs_[0].ks[0]));
+        TileBatch batch;
+        batch.n = kRateTasks;
+        for (int q = 0; q < kRateTasks; ++q)
+            batch.t[q] = TileTask{a, b, c + (size_t)q * T * T, T, T, T, T, T, T, 1.0, 1.0, 0, nullptr, 0, 0.0};
         float ms;
-        int rc = timed(0, devs_[0].ks[0], [&] { return launch_dgemm_tile(false, false, T, T, T, 1.0, a, T, b, T, 1.0, c, T, devs_[0].ks[0]); }, &ms);
+        int rc = timed(0, devs_[0].ks[0], [&] { return launch_dgemm_batch(false, false, batch, devs_[0].ks[0]); }, &ms);
         cudaFree(a);
         cudaFree(b);
         cudaFree(c);
         if (rc) return rc;
-        topo.rate_mflops = std::max<int64_t>(1, (int64_t)(2.0 * T * T * T / (ms * 1e3)));
+        topo.rate_mflops = std::max<int64_t>(1, (int64_t)(2.0 * T * T * T * kRateTasks / (ms * 1e3)));
     }
     for (int g = 0; g < G; ++g) {
         cudaSetDevice(devs_[g].phys);
@@ -438,13 +445,19 @@ int Runtime::probe_topology_rank() {
     // FP64 tile-task rate, measured by rank 0 for everyone (T <= 2048, in its arena)
     me.rate_mflops = 0;
     if (rank_ == 0 && cfg_.task_rate_mflops <= 0) {
+        // one grouped launch of up to 8 tile tasks, as in the single-process probe
         const int64_t T = std::min<int64_t>(flags_.T, 2048);
         const size_t tb = (size_t)T * T * 8;
-        if ((int64_t)(3 * tb) <= d.arena_bytes) {
+        const int nt = (int)std::min<int64_t>(8, d.arena_bytes / (int64_t)tb - 2);
+        if (nt >= 1) {
             double *a = reinterpret_cast<double *>(d.arena), *b = a + (size_t)T * T, *c = b + (size_t)T * T;
-            XK_CK(cudaMemsetAsync(d.arena, 0, 3 * tb, d.ks[0]));
-            if ((rc = timed(d.ks[0], [&] { return launch_dgemm_tile(false, false, T, T, T, 1.0, a, T, b, T, 1.0, c, T, d.ks[0]); }, &ms))) return rc;
-            me.rate_mflops = std::max<int64_t>(1, (int64_t)(2.0 * T * T * T / (ms * 1e3)));
+            XK_CK(cudaMemsetAsync(d.arena, 0, (2 + nt) * tb, d.ks[0]));
+            TileBatch batch;
+            batch.n = nt;
+            for (int q = 0; q < nt; ++q)
+                batch.t[q] = TileTask{a, b, c + (size_t)q * T * T, T, T, T, T, T, T, 1.0, 1.0, 0, nullptr, 0, 0.0};
+            if ((rc = timed(d.ks[0], [&] { return launch_dgemm_batch(false, false, batch, d.ks[0]); }, &ms))) return rc;
+            me.rate_mflops = std::max<int64_t>(1, (int64_t)(2.0 * T * T * T * nt / (ms * 1e3)));
         }
     }
     if (!sess_->barrier(300.0)) {

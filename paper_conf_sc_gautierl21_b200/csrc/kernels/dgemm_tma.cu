@@ -133,10 +133,13 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
     const int tiles_n = (int)((t.N + BN - 1) / BN);
     const int gm = batch.group_m > 0 ? batch.group_m : tiles_m;
     const int per_group = gm * tiles_n;
-    const int first = (local / per_group) * gm;
+    const int grp = local / per_group, first = grp * gm;
     const int gsz = min(tiles_m - first, gm);
     const int in_group = local % per_group;
-    const int m0 = (first + in_group % gsz) * BM, n0 = (in_group / gsz) * BN;
+    // snake: odd groups walk the n-blocks backwards, so the first CTAs of a group read the
+    // B panel the last CTAs of the previous group left in L2
+    const int nblk = (batch.snake && (grp & 1)) ? tiles_n - 1 - in_group / gsz : in_group / gsz;
+    const int m0 = (first + in_group % gsz) * BM, n0 = nblk * BN;
     const int64_t M = t.M, N = t.N;
     const int tri = t.tri;
     if ((tri == 1 && m0 + BM - 1 < n0) || (tri == 2 && n0 + BN - 1 < m0)) return;
@@ -361,6 +364,12 @@ cudaError_t launch_dgemm_tma(bool ta, bool tb, TmaBatch &b, cudaStream_t st) {
         group_m = (e && *e) ? atoi(e) : 16;
     }
     b.group_m = group_m;
+    static int snake = -1;
+    if (snake < 0) {
+        const char *e = getenv("XK_SNAKE");
+        snake = (e && *e == '0') ? 0 : 1;
+    }
+    b.snake = snake;
     constexpr size_t smem = STAGES * STAGE_BYTES + STAGES * 8 + STAGES * 4 + 1024;
     int total = 0;
     for (int q = 0; q < b.n; ++q) {

@@ -45,6 +45,7 @@ constexpr int kMaxTmaBatch = 16;
 struct TmaBatch {
     int n = 0;
     int group_m = 16;  // CTA raster: m-blocks per group (L2 reuse); 0 = column-major raster
+    int snake = 1;     // odd groups walk the n-blocks backwards (the B panel at a group boundary is reused)
     int cta_start[kMaxTmaBatch + 1] = {};
     TmaTask t[kMaxTmaBatch];
 };

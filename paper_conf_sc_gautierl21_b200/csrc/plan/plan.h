@@ -30,7 +30,7 @@ struct Topology {
 struct Flags {
     int topo = XK_TOPO_RANKED;
     int optimistic = 1;
-    int window = 2;
+    int window = 4;
     int P = 1, Q = 1;
     int64_t T = 2048;
     int64_t mem_bytes = 0;  // tile-cache capacity per GPU the plan must fit (0 = unlimited)

@@ -117,7 +117,7 @@ class Tile:
 
 
 class Model:
-    def __init__(self, bw, rate_mflops=35000000, topo="ranked", optimistic=True, window=2,
+    def __init__(self, bw, rate_mflops=35000000, topo="ranked", optimistic=True, window=4,
                  grid=(0, 0), tile=2048, mem_bytes=0):
         self.bw = [list(r) for r in bw]
         self.G = len(bw) - 1
