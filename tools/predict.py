@@ -15,7 +15,7 @@ boxes = {
     # (round-2 grouped launch, measured)
     "hgx_b200": (uniform(8, peer=700000, host=55000), 35800000),
 }
-out = {}
+out = {"params": {"window": 4, "note": "planner defaults (window W = 4, DESIGN.md Q17); the model's makespan is pinned to one-GPU measurements within 4% (profiles/r02_model_fidelity.jsonl), multi-GPU timing unpinned"}}
 for box, (bw, rate) in boxes.items():
     for N in (16384, 32768):
         T = 2048
