@@ -227,7 +227,9 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
     }
     cp_wait<0>();
 
-    // epilogue: D = alpha*acc + beta*C (C not read when beta == 0)
+    // epilogue: D = alpha*acc + beta*C (+ beta2*C2) (C, C2 not read when their beta is 0);
+    // one row fragment's loads are issued before its stores (see dgemm_tma.cu: interleaved,
+    // every element would cost an L2 round trip, since a store may alias a later load)
     const double alpha = t.alpha, beta = t.beta, beta2 = t.beta2;
     double *C = t.C;
     const int64_t ldc = t.ldc;
@@ -236,21 +238,27 @@ dgemm_tile_kernel(const __grid_constant__ TileBatch batch) {
 #pragma unroll
     for (int i = 0; i < MF; ++i) {
         const int64_t r = m0 + wm + i * 8 + fr;
-        if (r >= M) continue;
+        double cv[NF][2], c2v[NF][2];
 #pragma unroll
-        for (int j = 0; j < NF; ++j) {
+        for (int j = 0; j < NF; ++j)
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
                 const int64_t c = n0 + wn + j * 8 + fc * 2 + h;
-                if (c >= N) continue;
-                if ((tri == 1 && r < c) || (tri == 2 && r > c)) continue;
-                double *p = C + r + c * ldc;
-                double v = alpha * acc[i][j][h];
-                if (beta != 0.0) v = fma(beta, *p, v);
-                if (beta2 != 0.0) v = fma(beta2, C2[r + c * ldc2], v);
-                *p = v;
+                const bool ok = r < M && c < N && !((tri == 1 && r < c) || (tri == 2 && r > c));
+                cv[j][h] = (ok && beta != 0.0) ? C[r + c * ldc] : 0.0;
+                c2v[j][h] = (ok && beta2 != 0.0) ? C2[r + c * ldc2] : 0.0;
             }
-        }
+#pragma unroll
+        for (int j = 0; j < NF; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int64_t c = n0 + wn + j * 8 + fc * 2 + h;
+                if (r >= M || c >= N || (tri == 1 && r < c) || (tri == 2 && r > c)) continue;
+                double v = alpha * acc[i][j][h];
+                if (beta != 0.0) v = fma(beta, cv[j][h], v);
+                if (beta2 != 0.0) v = fma(beta2, c2v[j][h], v);
+                C[r + c * ldc] = v;
+            }
     }
 }
 
