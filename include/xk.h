@@ -107,7 +107,7 @@ typedef struct xk_config {
 } xk_config_t;
 
 /* Fill *cfg with defaults, then apply the environment (XK_NGPUS, XK_TILE,
- * XK_TOPO=ranked|unranked|home, XK_OPTIMISTIC=0|1, XK_WINDOW, XK_KSTREAMS, XK_PROBE). */
+ * XK_TOPO=ranked|unranked|home, XK_OPTIMISTIC=0|1, XK_WINDOW, XK_KSTREAMS, XK_PROBE, XK_TASK_RATE). */
 void xk_config_default(xk_config_t *cfg);
 
 /* ------------------------------------------------------------------ lifecycle */

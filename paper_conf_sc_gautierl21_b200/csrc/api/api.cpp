@@ -115,6 +115,8 @@ void xk_config_default(xk_config_t *cfg) {
     cfg->window = env_int("XK_WINDOW", 4);
     cfg->kstreams = env_int("XK_KSTREAMS", 2);
     cfg->probe = env_int("XK_PROBE", 1);
+    const char *rate = std::getenv("XK_TASK_RATE");  // planner task rate in MFLOP/s (0 = measured)
+    cfg->task_rate_mflops = (rate && *rate) ? std::atoll(rate) : 0;
 }
 
 int xk_init(const xk_config_t *cfg) {

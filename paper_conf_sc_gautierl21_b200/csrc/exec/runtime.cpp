@@ -639,8 +639,9 @@ int Runtime::issue(const Rec &R) {
         set_error("rank mode: more plan records in flight than the completion-flag ring holds");
         return XK_ERR_UNSUPPORTED;
     }
+    const int max_batch = planner_->batch_hint() > 0 ? std::min(max_batch_, planner_->batch_hint()) : max_batch_;
     if (defer_d2h_ && here(r) && r.kind == XK_REC_D2H && r.dep[0] >= 0 && batch_[r.src].contains_seq(r.dep[0]) &&
-        batch_[r.src].recs.back().remaining >= max_batch_) {
+        batch_[r.src].recs.back().remaining >= max_batch) {
         PendingBatch &bt = batch_[r.src];
         bt.deferred.push_back(R);
         bt.in_ids.push_back((int64_t)R.key * XK_MAX_GPUS + r.src);
@@ -727,7 +728,7 @@ int Runtime::issue(const Rec &R) {
                              bt.recs[0].side != R.side || bt.recs[0].uplo != R.uplo || bt.recs[0].ta != R.ta ||
                              bt.recs[0].diag != R.diag ||
                              (R.side == 'L' ? bt.recs[0].m != R.m : bt.recs[0].n != R.n));
-            conflict = conflict || (int)bt.recs.size() >= max_batch_ || bt.touches(idO, true) ||
+            conflict = conflict || (int)bt.recs.size() >= max_batch || bt.touches(idO, true) ||
                        bt.touches(idA, false) || (idC2 >= 0 && bt.touches(idC2, false));
             for (int q = 0; q < 4 && !conflict; ++q)
                 if (r.dep[q] >= 0 && bt.contains_seq(r.dep[q])) conflict = true;
@@ -809,7 +810,7 @@ int Runtime::issue(const Rec &R) {
         // ... and ramps down (half of the GPU's remaining tasks) at the end, so the write-back
         // of the last C tiles does not wait for one large final batch
         const int64_t left0 = (bt.recs.empty() ? R.remaining : bt.recs[0].remaining) + 1;
-        const int cap = (int)std::min<int64_t>(std::min<int64_t>(max_batch_, std::max<int64_t>(1, (left0 + 1) / 2)),
+        const int cap = (int)std::min<int64_t>(std::min<int64_t>(max_batch, std::max<int64_t>(1, (left0 + 1) / 2)),
                                                (int64_t)1 << std::min<int64_t>(batches_in_call_[g] / ramp_div_, 5));
         bool conflict = (int)bt.recs.size() >= cap ||
                         (!bt.recs.empty() && (bt.op == XK_OP_TRSM_DIAG || bt.op == XK_OP_TRMM_DIAG)) ||

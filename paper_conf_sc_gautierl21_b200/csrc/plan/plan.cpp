@@ -1085,6 +1085,10 @@ int Planner::plan_trxm(const xk_call_t &c, bool solve, std::vector<Rec> &out, st
             b_on_gpus = cur;
         }
     const int64_t Dw = b_on_gpus ? nsteps : 2 * (left ? std::min(flags_.P, flags_.Q) : std::max(flags_.P, flags_.Q));
+    // executor batch cap (reading R19): the R10 window turns a TRSM step's catch-up updates
+    // into per-tile chains, and TRMM's contributions are per-tile chains, so consecutive
+    // 16-task batches would depend on each other and could not overlap on the kernel streams
+    batch_hint_ = solve ? (b_on_gpus ? 0 : 4) : 8;
     // TRMM from the host (reading R15): every step reads B's input tiles from a
     // per-call shadow, so no GEMM reads a tile the sweep overwrites and the sweep runs in the
     // solve direction (top-down for left/lower): step s needs one new row (column) of B
@@ -1430,6 +1434,7 @@ void Planner::emit(const Rec &R, std::vector<Rec> &out) {
 int Planner::plan(const xk_call_t &c, std::vector<Rec> &out, std::string &err, const Sink *sink) {
     sink_ = sink;
     sink_rc_ = 0;
+    batch_hint_ = 0;
     int rc = plan_impl(c, out, err);
     sink_ = nullptr;
     if (rc == XK_OK && sink_rc_) rc = sink_rc_;

@@ -105,6 +105,9 @@ public:
     const Entry &entry(int id) const { return entries_[id]; }
     const Matrix &matrix(int id) const { return mats_[id]; }
     int G() const { return topo_.G; }
+    // Grouped-launch cap the current call's task structure suits (0 = the executor's
+    // default): set before the call's first record is emitted (R19).
+    int batch_hint() const { return batch_hint_; }
     int owner(int64_t i, int64_t j) const {
         return (int)((i % flags_.P) * flags_.Q + (j % flags_.Q));
     }
@@ -136,6 +139,7 @@ public:
     int link_class(int s, int d) const { return cls_[(size_t)s * (topo_.G + 1) + d]; }
 
 private:
+    int batch_hint_ = 0;
     struct Input { int key; int64_t ver; int operand; int cnt = -1; };  // cnt: readers slot
     struct Inputs {  // at most 4 inputs per task, no heap allocation
         Input v[4];
