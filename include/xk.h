@@ -235,6 +235,8 @@ typedef struct xk_stats {
     int64_t plan_records_local;      /* ... of which executed by this process (rank mode: its GPU) */
     double host_issue_ms;            /* host wall time planning + issuing them (the per-call
                                         "creation and scheduling of dynamic tasks") */
+    int64_t device_allocs;           /* new device tile buffers (not served by the free lists) */
+    double device_alloc_ms;          /* host wall time spent obtaining them */
 } xk_stats_t;
 /* Counters since xk_init / the last xk_reset_stats: the per-link byte counts are the paper's
  * transfer breakdown (SecIV-E) and the evidence that the heuristics cut PCIe bytes

@@ -215,7 +215,7 @@ def get_stats():
         out[f] = list(getattr(st, f))[:G]
     for f in ("forwards_inflight", "forwards_valid", "kernel_launches", "host_registrations",
               "kernel_ms_total", "kernel_timed_launches", "kernel_timed_flops", "plan_records",
-              "plan_records_local", "host_issue_ms"):
+              "plan_records_local", "host_issue_ms", "device_allocs", "device_alloc_ms"):
         out[f] = getattr(st, f)
     out["trace_ms"] = dict(zip(("h2d", "p2p", "kernel", "d2h"), list(st.trace_ms)))
     out["link_bytes"] = [[st.link_bytes[s * (G + 1) + d] for d in range(G + 1)] for s in range(G + 1)]

@@ -51,7 +51,7 @@ class Stats(ctypes.Structure):
                 ("kernel_timed_launches", i64), ("kernel_timed_flops", i64),
                 ("link_bytes", i64 * ((MAX_GPUS + 1) * (MAX_GPUS + 1))),
                 ("trace_ms", c_double * 4), ("plan_records", i64), ("plan_records_local", i64),
-                ("host_issue_ms", c_double)]
+                ("host_issue_ms", c_double), ("device_allocs", i64), ("device_alloc_ms", c_double)]
 
 
 class Topo(ctypes.Structure):

@@ -573,6 +573,15 @@ double *Runtime::alloc(int g, size_t bytes, int *rc) {
         return reinterpret_cast<double *>(d.arena + off);
     }
     if ((*rc = set_dev(g))) return nullptr;
+    const auto t_alloc = std::chrono::steady_clock::now();
+    struct AllocTimer {  // counts the new buffer and its host time on every exit path
+        xk_stats_t &st;
+        std::chrono::steady_clock::time_point t0;
+        ~AllocTimer() {
+            st.device_allocs++;
+            st.device_alloc_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        }
+    } alloc_timer{stats, t_alloc};
     double *p = nullptr;
     cudaError_t e = cudaMalloc(&p, bytes);
     if (e != cudaSuccess) {

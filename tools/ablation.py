@@ -60,6 +60,11 @@ for name, topo, opt in [m for m in MODES if not ONLY or m[0] in ONLY]:
         for X in (A, B, C, L):
             xk.memory_prefetch_async(N, N, X, N)
         xk.sync()
+        # a discarded data-on-device warm-up call too: the first one allocates the
+        # forwarded tiles' device buffers (316 cudaMalloc for DTRSM N=32768 on 8 logical GPUs,
+        # up to ~1 s of host time), which the host-resident warm-up above does not cover
+        call(True)
+        xk.sync()
     xk.reset_stats()
     torch.cuda.synchronize()
     t0 = time.perf_counter()

@@ -1,6 +1,7 @@
 #!/bin/bash
 # A/B of the GEMM epilogue: loads batched per row fragment (EPI_ROWS=1, default), per two
-# (EPI_ROWS=2), and the previous interleaved load/store epilogue (tools/_ab/dgemm_tma_old.cu)
+# (EPI_ROWS=2), and the previous interleaved load/store epilogue (tools/_ab/dgemm_tma_old.cu =
+# the parent commit's dgemm_tma.cu, extracted before the run)
 mkdir -p gpurun_out
 K=paper_conf_sc_gautierl21_b200/csrc/kernels/dgemm_tma.cu
 cp $K /tmp/dgemm_tma_new.cu

@@ -65,6 +65,9 @@ def call_async():
     xk.sync()
 
 
+if DOD and os.environ.get("SYNC_WARMUP") == "1":  # the ablation's sequence: a sync call first
+    call()
+    torch.cuda.synchronize()
 if DOD:
     for X in (A, B, C, L):
         xk.memory_prefetch_async(N, N, X, N)
