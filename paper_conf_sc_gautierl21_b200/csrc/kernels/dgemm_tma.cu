@@ -43,6 +43,9 @@ constexpr int STAGES = 4;
 #define XK_EPI_ROWS 1
 #endif
 constexpr int EPI_ROWS = XK_EPI_ROWS;  // row fragments per epilogue load batch
+#ifndef XK_FB1
+#define XK_FB1 1  // single-buffered B fragments (0: double-buffered, the round-2 A/B baseline)
+#endif
 static_assert((WM / 8) % EPI_ROWS == 0, "epilogue chunking");
 constexpr int A_BYTES = BM * BK * 8, B_BYTES = BN * BK * 8, STAGE_BYTES = A_BYTES + B_BYTES;
 
@@ -192,6 +195,25 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
     for (int i = 0; i < MF; ++i)
 #pragma unroll
         for (int j = 0; j < NF; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+#if XK_FB1
+    // B fragments single-buffered (loaded right before their DMMAs; the other warps of the
+    // scheduler cover the shared-load latency), A fragments double-buffered
+    double fa[2][MF], fb[1][NF];
+    auto load_b = [&](int stage, int s) {
+        const unsigned char *sb = sgen + stage * STAGE_BYTES + A_BYTES;
+        const int x = (s & 1) | ((s & 2) << 1);
+#pragma unroll
+        for (int j = 0; j < NF; ++j)
+            fb[0][j] = *reinterpret_cast<const double *>(sb + (laneB ^ const_part<B_MN>(wn + j * 8, x)));
+    };
+    auto load_frags = [&](int buf, int stage, int s) {
+        const unsigned char *sa = sgen + stage * STAGE_BYTES;
+        const int x = (s & 1) | ((s & 2) << 1);
+#pragma unroll
+        for (int i = 0; i < MF; ++i)
+            fa[buf][i] = *reinterpret_cast<const double *>(sa + (laneA ^ const_part<A_MN>(wm + i * 8, x)));
+    };
+#else
     double fa[2][MF], fb[2][NF];
     auto load_frags = [&](int buf, int stage, int s) {
         const unsigned char *sa = sgen + stage * STAGE_BYTES;
@@ -204,6 +226,7 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
         for (int j = 0; j < NF; ++j)
             fb[buf][j] = *reinterpret_cast<const double *>(sb + (laneB ^ const_part<B_MN>(wn + j * 8, x)));
     };
+#endif
 
     mbar_wait(full(0), 0);
     load_frags(0, 0, 0);
@@ -235,6 +258,9 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
 #pragma unroll
         for (int s = 0; s < BK / 4; ++s) {
             const int cur = s & 1;
+#if XK_FB1
+            load_b(st, s);
+#endif
             if (s + 1 < BK / 4) {
                 load_frags(cur ^ 1, st, s + 1);
                 if (s + 2 == BK / 4) {
@@ -267,7 +293,7 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
 #pragma unroll
             for (int i = 0; i < MF; ++i)
 #pragma unroll
-                for (int j = 0; j < NF; ++j) dmma(acc[i][j], fa[cur][i], fb[cur][j]);
+                for (int j = 0; j < NF; ++j) dmma(acc[i][j], fa[cur][i], fb[XK_FB1 ? 0 : cur][j]);
         }
     }
 
