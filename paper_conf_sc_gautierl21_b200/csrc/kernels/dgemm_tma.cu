@@ -255,36 +255,41 @@ __global__ void __launch_bounds__(NTHREADS, 2) dgemm_tma_kernel(const __grid_con
                 }
             }
         }
+        // this warp's last read of stage st is done; the last warp to get here refills the
+        // stage with block kb + STAGES (no CTA-wide barrier, no dedicated producer warp).
+        // The count is an acq_rel RMW: each warp's increment releases its reads of the stage
+        // (ordered before lane 0's RMW by __syncwarp), and the last increment acquires all of
+        // them (one release sequence), so the refill's async-proxy TMA write (after
+        // fence.proxy.async) follows every read.
+        auto release_stage = [&]() {
+            __syncwarp();
+            if (lane == 0) {
+                uint32_t old;
+                asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;\n"
+                             : "=r"(old) : "r"(smem_u32(&done_cnt[st])) : "memory");
+                if (old == NWARPS - 1) {
+                    atomicExch(&done_cnt[st], 0);
+                    if (kb + STAGES < KB) {
+                        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+                        produce(kb + STAGES);
+                    }
+                }
+            }
+        };
 #pragma unroll
         for (int s = 0; s < BK / 4; ++s) {
             const int cur = s & 1;
 #if XK_FB1
             load_b(st, s);
+            // the last step's B fragments are this warp's last read of the stage (its A
+            // fragments were loaded one step earlier)
+            if (s + 1 == BK / 4) release_stage();
 #endif
             if (s + 1 < BK / 4) {
                 load_frags(cur ^ 1, st, s + 1);
-                if (s + 2 == BK / 4) {
-                    // this warp's last read of the stage is done; the last warp to get here
-                    // refills the stage with block kb + STAGES (no CTA-wide barrier, no
-                    // dedicated producer warp)
-                    // The count is an acq_rel RMW: each warp's increment releases its reads
-                    // of the stage (ordered before lane 0's RMW by __syncwarp), and the last
-                    // increment acquires all of them (one release sequence), so the refill's
-                    // async-proxy TMA write (after fence.proxy.async) follows every read.
-                    __syncwarp();
-                    if (lane == 0) {
-                        uint32_t old;
-                        asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;\n"
-                                     : "=r"(old) : "r"(smem_u32(&done_cnt[st])) : "memory");
-                        if (old == NWARPS - 1) {
-                            atomicExch(&done_cnt[st], 0);
-                            if (kb + STAGES < KB) {
-                                asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-                                produce(kb + STAGES);
-                            }
-                        }
-                    }
-                }
+#if !XK_FB1
+                if (s + 2 == BK / 4) release_stage();  // the next step's A and B are loaded
+#endif
             } else if (kb + 1 < KB) {
                 const int nx = (kb + 1) % STAGES;
                 mbar_wait(full(nx), (uint32_t)(((kb + 1) / STAGES) & 1));
