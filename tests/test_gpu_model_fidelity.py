@@ -5,7 +5,7 @@ grouped-launch task rate the runtime measures at xk_init.  Its byte counts are p
 elsewhere; here its makespan is compared with the wall time of the same synchronous
 host-resident call on one GPU -- the configuration whose resources (one compute engine, one
 H2D and one D2H link) are the model's own.  Measured with the default window W = 4 on a B200:
-predicted / measured time 0.96-1.04 over every routine at N = 32768 and DGEMM at N = 16384
+predicted / measured time 1.01-1.08 over every routine at N = 32768 and DGEMM at N = 16384
 (profiles/r02_model_fidelity.jsonl); the bound below leaves room for box-to-box variation.
 """
 import time
